@@ -1,0 +1,165 @@
+/*
+ * spline_builder.h -- C ABI of the B200-native batched spline-coefficient
+ * builder (PAPER.md: Asahi et al., "Development of performance portable
+ * spline solver for exa-scale plasma turbulence simulation", SC'24-W).
+ *
+ * The problem (Sec. II.B, Eq. 2): one B-spline collocation
+ * matrix A, fixed in time, solved against a huge batch of right-hand sides
+ * b ("a fixed single matrix A and multiple right-hand sides"), in place
+ * ("b stores the right-hand side vectors on entry and stores the solution
+ * vectors on exit").  A is factored once at create time on the host
+ * with the Schur-complement block split of Eq. 3-4,
+ * and every solve runs Algorithm 1 in one fused sm_100a kernel:
+ *   x0' = Q^{-1} b0            (banded LDL^T / LU: pttrs, pbtrs or gbtrs, Table I)
+ *   x1  = delta'^{-1} (b1 - lambda x0')   (COO spmv + getrs)
+ *   x0  = x0' - beta x1                     (COO spmv, beta = Q^{-1} gamma)
+ *
+ * All functions are extern "C", take plain pointers and sizes, and never
+ * throw.  No torch type appears here.  Status codes are the SB_* values
+ * below; the message of the last failure on the calling thread is returned
+ * by spline_builder_last_error().
+ */
+#ifndef SPLINE_BUILDER_H
+#define SPLINE_BUILDER_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct spline_builder *spline_builder_t; /* opaque, immutable after create */
+
+/* boundary conditions (PAPER.md P:55 periodic; non-periodic per BASELINE C3) */
+enum { SB_PERIODIC = 0, SB_GREVILLE = 1, SB_HERMITE = 2 };
+/* element types of the right-hand sides */
+enum { SB_F64 = 0, SB_F32 = 1 };
+/* status codes */
+enum {
+    SB_OK = 0,
+    SB_INVALID_ARG = 1, /* bad argument; nothing was launched                 */
+    SB_SINGULAR = 2,    /* A (or Q / delta') could not be factored             */
+    SB_CUDA = 3,        /* a CUDA runtime / driver call or launch failed       */
+    SB_NOMEM = 4,       /* host or device allocation failed                    */
+    SB_UNSUPPORTED = 5  /* valid request outside what this build implements   */
+};
+/* create flags */
+enum {
+    SB_FLAG_HOST_ONLY = 1 /* factor on the host only; no device upload (solve_* then
+                             return SB_UNSUPPORTED).  For inspection / CPU tests. */
+};
+
+/*
+ * spline_builder_create -- one-time construction and factorisation
+ * ("the factorization is only done once at
+ * initialization ... and copy the result to the device").
+ *
+ *   degree   spline degree p, 1..5.
+ *   n_points number of interpolation conditions, which fixes the number of
+ *            cells N:   periodic  N = n_points          (nbasis n = N)
+ *                       Greville  N = n_points - p      (n = N + p)
+ *                       Hermite   N = n_points - 1 (odd p) or N = n_points
+ *                                 (even p, values at cell midpoints); n = N + p
+ *   bc       SB_PERIODIC, SB_GREVILLE or SB_HERMITE (both ends alike).
+ *   knots    NULL -> uniform mesh on [0, 1] (all cells of width 1/N exactly);
+ *            else N+1 strictly increasing breakpoints (host pointer, read
+ *            during the call only; the periodic period is knots[N]-knots[0]).
+ *
+ * Row order of every right-hand side (length n):
+ *   periodic / Greville: b_j = f(xi_j), xi_j the Greville abscissa of basis j
+ *     (periodic basis j is centred on xi_j; uniform: xi_j = x_j for odd p,
+ *     x_j + h/2 for even p).
+ *   Hermite: [f^(1..nbc)(x_0), f(x_0) ... f(x_N), f^(1..nbc)(x_N)] with raw
+ *     derivatives (odd p, nbc = (p-1)/2); even p: values at the N cell
+ *     midpoints, nbc = p/2.
+ * The handle owns host and device copies of the factors on the CUDA device
+ * current at the call.  Returns NULL on failure (see last_error / the
+ * status in spline_builder_last_status()).
+ */
+spline_builder_t spline_builder_create(int degree, int n_points, int bc, const double *knots);
+
+/* Same as create, with an explicit Schur split: the delta index set is the
+ * first split_lo and the last split_hi rows/columns of A.
+ * split_lo = split_hi = -1 selects the default.  Periodic requires
+ * split_lo = 0 and split_hi >= the circulant half-bandwidth (or -1). */
+spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, const double *knots,
+                                          int split_lo, int split_hi, int flags);
+
+/*
+ * spline_builder_solve -- in-place batched solve of fp64 right-hand sides
+ * (Algorithm 1; fused kernel of Listing 6).
+ *
+ *   rhs           DEVICE pointer on the handle's device, caller owned.  On
+ *                 entry b, on exit the spline coefficients x (same layout).
+ *   batch         number of right-hand sides (>= 0; 0 is a no-op).
+ *   batch_stride  elements between consecutive right-hand sides:
+ *                   1   -> batch-contiguous (the paper's layout, P:143,
+ *                          P:391): element (row j, rhs r) at rhs[j*batch + r]
+ *                   >=n -> point-contiguous: element (j, r) at
+ *                          rhs[r*batch_stride + j]   (GYSELA slice, C4)
+ *                 anything else -> SB_INVALID_ARG (use _strided).
+ *   stream        cudaStream_t (NULL = legacy default stream) on which the
+ *                 kernel is enqueued; the call is asynchronous.
+ * Concurrent solves on different streams with one handle are allowed.
+ */
+int spline_builder_solve(spline_builder_t h, double *rhs, int64_t batch, int64_t batch_stride, void *stream);
+
+/* fp32 storage, same semantics (compute in fp32). */
+int spline_builder_solve_f32(spline_builder_t h, float *rhs, int64_t batch, int64_t batch_stride, void *stream);
+
+/* General strided layout: element (row j, rhs r) at
+ * rhs[r*batch_stride + j*point_stride]; dtype SB_F64 or SB_F32.  Strides
+ * in elements, > 0, and the (j, r) -> offset map must be one-to-one. */
+int spline_builder_solve_strided(spline_builder_t h, void *rhs, int dtype, int64_t batch, int64_t batch_stride,
+                                 int64_t point_stride, void *stream);
+
+/*
+ * spline_builder_solve_host -- end-to-end solve of HOST data (fp64 or fp32,
+ * batch-contiguous (n, batch) layout with leading dimension ld >= batch):
+ * the batch is cut into chunks that are copied host->device, solved and
+ * copied back on a pipeline of streams so that the copies overlap the
+ * kernels.  host_rhs should be pinned (cudaHostRegister / cudaMallocHost)
+ * for full PCIe bandwidth.  Synchronous: returns when the data is back.
+ */
+int spline_builder_solve_host(spline_builder_t h, void *host_rhs, int dtype, int64_t batch, int64_t ld);
+
+void spline_builder_destroy(spline_builder_t h); /* caller syncs first; NULL ok */
+
+/* ------------------------------------------------------------ queries */
+typedef struct {
+    int degree, bc, n_cells, nbasis;
+    int split_lo, split_hi, k;      /* delta' is k x k, k = split_lo + split_hi */
+    int q_kl, q_ku;                 /* band of Q (Table I type below)            */
+    int q_type;                     /* 0 pttrs (sym tridiag), 1 pbtrs (sym band),
+                                       2 gbtrs (general band, no interchanges)   */
+    int nnz_lambda, nnz_beta;       /* COO sizes; beta kept if > 1e-14   */
+    int beta_rows_head, beta_rows_tail; /* Q rows at each end touched by beta     */
+    int n_segments, seg_len;        /* in-CTA segment split of the Q recurrences  */
+    int carry_fwd, carry_bwd;       /* predecessor segments in the carry walks    */
+    double max_pivot_growth;        /* max |U| / max |Q| of the no-pivot LU        */
+} spline_builder_info_t;
+
+int spline_builder_get_info(spline_builder_t h, spline_builder_info_t *info);
+int64_t spline_builder_nbasis(spline_builder_t h);
+
+/* Host copies of the Schur blocks for inspection (any pointer may be NULL):
+ * lambda COO (rows in [0,k), cols in [0,n-k)) and beta COO (rows in
+ * [0,n-k), cols in [0,k)), indices are delta-/Q-local; delta' (k*k,
+ * row-major, before LU).  Arrays must hold nnz / k*k entries. */
+int spline_builder_get_blocks(spline_builder_t h, int *lam_rows, int *lam_cols, double *lam_vals, int *beta_rows,
+                              int *beta_cols, double *beta_vals, double *delta_prime);
+
+/* Host-side fp64 reference solve of the SAME factorisation (Algorithm 1 on
+ * the CPU, serial).  Used by create's self-check; exported for tests of the
+ * host plan.  Layout as spline_builder_solve_strided. */
+int spline_builder_solve_cpu_plan(spline_builder_t h, double *rhs, int64_t batch, int64_t batch_stride,
+                                  int64_t point_stride);
+
+const char *spline_builder_last_error(void); /* thread-local; never NULL */
+int spline_builder_last_status(void);        /* status of the last failed call */
+const char *spline_builder_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPLINE_BUILDER_H */

@@ -1,0 +1,158 @@
+"""B200-native batched spline-coefficient builder.
+
+Python face of ``include/spline_builder.h``: :class:`SplineBuilder` wraps one
+handle (one collocation matrix, factored once at create) and
+solves batches of right-hand sides in place on the GPU (Algorithm 1,
+P:86-91).  torch is used only for device memory and streams; the names
+mirror the C ABI and every call is argument marshalling into
+``libsplinebuilder.so``.
+"""
+from __future__ import annotations
+
+import ctypes
+
+from . import _lib
+from ._lib import (SB_F32, SB_F64, SB_FLAG_HOST_ONLY, SB_GREVILLE, SB_HERMITE, SB_PERIODIC, SplineBuilderError,
+                   SplineBuilderInfo)
+
+PERIODIC, GREVILLE, HERMITE = SB_PERIODIC, SB_GREVILLE, SB_HERMITE
+
+__all__ = ["SplineBuilder", "SplineBuilderError", "PERIODIC", "GREVILLE", "HERMITE", "load_library"]
+
+
+def load_library():
+    """Load the native library (raises ImportError if it was not built)."""
+    return _lib.load()
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return ctypes.c_void_p(stream)
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+class SplineBuilder:
+    """One spline space (degree, points, boundary condition, breakpoints).
+
+    ``split`` = (split_lo, split_hi) forces the Schur split of Eq. 3
+    (default: chosen at create).  ``host_only`` factors without touching the
+    GPU (inspection / CPU tests)."""
+
+    def __init__(self, degree: int, n_points: int, bc: int = PERIODIC, knots=None, split=None,
+                 host_only: bool = False):
+        lib = _lib.load()
+        self._lib = lib
+        kbuf = None
+        if knots is not None:
+            import numpy as np
+            self._knots = np.ascontiguousarray(knots, dtype=np.float64)
+            kbuf = ctypes.c_void_p(self._knots.ctypes.data)
+        lo, hi = (-1, -1) if split is None else split
+        flags = SB_FLAG_HOST_ONLY if host_only else 0
+        h = lib.spline_builder_create_ex(int(degree), int(n_points), int(bc), kbuf, int(lo), int(hi), flags)
+        if not h:
+            raise SplineBuilderError(lib.spline_builder_last_status(), _lib.last_error())
+        self._h = ctypes.c_void_p(h)
+        self.degree, self.n_points, self.bc = degree, n_points, bc
+        self.n = int(lib.spline_builder_nbasis(self._h))
+
+    # ------------------------------------------------------------ lifetime
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.spline_builder_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # ------------------------------------------------------------- queries
+    def info(self) -> dict:
+        inf = SplineBuilderInfo()
+        _lib.check(self._lib.spline_builder_get_info(self._h, ctypes.byref(inf)))
+        return inf.as_dict()
+
+    def blocks(self):
+        """(lambda COO, beta COO, delta') as numpy arrays (host copies)."""
+        import numpy as np
+        inf = self.info()
+        k, nl, nb = inf["k"], inf["nnz_lambda"], inf["nnz_beta"]
+        lr, lc, lv = np.empty(nl, np.int32), np.empty(nl, np.int32), np.empty(nl)
+        br, bc, bv = np.empty(nb, np.int32), np.empty(nb, np.int32), np.empty(nb)
+        dp = np.empty((k, k))
+        p = lambda a: ctypes.c_void_p(a.ctypes.data)  # noqa: E731
+        _lib.check(self._lib.spline_builder_get_blocks(self._h, p(lr), p(lc), p(lv), p(br), p(bc), p(bv), p(dp)))
+        return (lr, lc, lv), (br, bc, bv), dp
+
+    # -------------------------------------------------------------- solves
+    def solve_(self, rhs, batch_stride: int | None = None, stream=None):
+        """In-place solve of a CUDA tensor (fp64 or fp32).  Layouts:
+        (n, batch) contiguous -> batch-contiguous; (batch, n) contiguous ->
+        point-contiguous.  Anything else: :meth:`solve_strided_`."""
+        import torch
+        if not rhs.is_cuda:
+            raise ValueError("rhs must be a CUDA tensor (use solve_host for host data)")
+        if rhs.dtype not in (torch.float64, torch.float32):
+            raise TypeError("rhs must be float64 or float32")
+        if rhs.dim() != 2 or not rhs.is_contiguous():
+            raise ValueError("rhs must be a contiguous 2-D tensor")
+        if batch_stride is None:
+            if rhs.shape[0] == self.n:
+                batch, bs = rhs.shape[1], 1
+            elif rhs.shape[1] == self.n:
+                batch, bs = rhs.shape[0], self.n
+            else:
+                raise ValueError(f"no dimension of size n={self.n}")
+        else:
+            bs = batch_stride
+            batch = rhs.shape[1] if bs == 1 else rhs.shape[0]
+        fn = self._lib.spline_builder_solve if rhs.dtype == torch.float64 else self._lib.spline_builder_solve_f32
+        _lib.check(fn(self._h, ctypes.c_void_p(rhs.data_ptr()), int(batch), int(bs), _stream_handle(stream)))
+        return rhs
+
+    def solve_strided_(self, rhs, batch: int, batch_stride: int, point_stride: int, stream=None):
+        import torch
+        dt = SB_F64 if rhs.dtype == torch.float64 else SB_F32
+        _lib.check(self._lib.spline_builder_solve_strided(self._h, ctypes.c_void_p(rhs.data_ptr()), dt, int(batch),
+                                                          int(batch_stride), int(point_stride),
+                                                          _stream_handle(stream)))
+        return rhs
+
+    def solve_host_(self, arr, ld: int | None = None):
+        """End-to-end solve of host memory (numpy array or CPU tensor of shape
+        (n, >=batch), row-major).  Pinned memory gives full PCIe bandwidth."""
+        try:
+            import torch
+            is_t = isinstance(arr, torch.Tensor)
+        except ImportError:  # pragma: no cover
+            is_t = False
+        if is_t:
+            dt = SB_F64 if arr.dtype == torch.float64 else SB_F32
+            ptr, batch, ld0 = arr.data_ptr(), arr.shape[1], arr.stride(0)
+        else:
+            import numpy as np
+            dt = SB_F64 if arr.dtype == np.float64 else SB_F32
+            ptr, batch, ld0 = arr.ctypes.data, arr.shape[1], arr.strides[0] // arr.itemsize
+        _lib.check(self._lib.spline_builder_solve_host(self._h, ctypes.c_void_p(ptr), dt, int(batch),
+                                                       int(ld if ld is not None else ld0)))
+        return arr
+
+    def solve_cpu_plan_(self, arr):
+        """Host fp64 run of the same factorisation (create's self-check path;
+        for tests of the host plan only, not a product solve path)."""
+        import numpy as np
+        assert arr.dtype == np.float64 and arr.flags.c_contiguous and arr.shape[0] == self.n
+        _lib.check(self._lib.spline_builder_solve_cpu_plan(self._h, ctypes.c_void_p(arr.ctypes.data),
+                                                           int(arr.shape[1]), 1, int(arr.shape[1])))
+        return arr

@@ -1,0 +1,324 @@
+// capi.cpp -- the extern "C" boundary declared in include/spline_builder.h.
+// Host create (plan.cpp) + one packed device upload + kernel dispatch
+// (solve_kernels.cu).  No exception crosses the ABI.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/spline_builder.h"
+#include "device.hpp"
+#include "host/plan.hpp"
+
+namespace {
+
+thread_local std::string g_err = "";
+thread_local int g_status = 0;
+
+int fail(int code, const std::string &msg) {
+    g_err = msg;
+    g_status = code;
+    return code;
+}
+
+constexpr int LMAX_SEG = 32;  // must match the kernels' register segment length
+
+}  // namespace
+
+struct spline_builder {
+    sb::Plan plan;
+    int device = -1;
+    int num_sms = 0;
+    bool host_only = false;
+    void *blob = nullptr;  // device constants
+    size_t blob_bytes = 0;
+    sb::DevPlan dp{};
+    // staging for solve_host
+    std::mutex host_mu;
+    void *stage[3] = {nullptr, nullptr, nullptr};
+    size_t stage_bytes = 0;
+    cudaStream_t streams[3] = {nullptr, nullptr, nullptr};
+};
+
+namespace {
+
+struct Packer {
+    std::vector<unsigned char> bytes;
+    size_t add(const void *src, size_t n) {
+        size_t off = (bytes.size() + 15) / 16 * 16;
+        bytes.resize(off + (n + 15) / 16 * 16, 0);
+        if (n) std::memcpy(bytes.data() + off, src, n);
+        return off;
+    }
+    template <typename T>
+    size_t addv(const std::vector<T> &v) { return add(v.data(), v.size() * sizeof(T)); }
+};
+
+template <typename C>
+std::vector<C> conv(const std::vector<double> &v) {
+    return std::vector<C>(v.begin(), v.end());
+}
+
+int upload(spline_builder *h) {
+    const sb::Plan &P = h->plan;
+    const int K = P.K, nQ = P.nQ, k = P.k, W = P.Wh + P.Wt;
+    const int FS = 2 * K, BS = 2 * K + 2;
+    std::vector<double> fwd((size_t)nQ * FS, 0.0), bwd((size_t)nQ * BS, 0.0);
+    for (int i = 0; i < nQ; ++i) {
+        for (int m = 0; m < K; ++m) {
+            fwd[(size_t)i * FS + m] = P.Lb[(size_t)i * K + m];
+            fwd[(size_t)i * FS + K + m] = P.gspk[(size_t)i * K + m];
+            bwd[(size_t)i * BS + 1 + m] = P.Ub[(size_t)i * K + m];
+            bwd[(size_t)i * BS + 1 + K + m] = P.hspk[(size_t)i * K + m];
+        }
+        bwd[(size_t)i * BS] = P.dinv[i];
+    }
+    // dense thresholded beta rows over the head/tail windows (COO semantic)
+    std::vector<double> betaW((size_t)W * k, 0.0);
+    for (size_t e = 0; e < P.beta_v.size(); ++e) {
+        int slot = P.win_slot(P.beta_r[e]);
+        if (slot < 0) return fail(SB_UNSUPPORTED, "internal: beta row outside window");
+        betaW[(size_t)slot * k + P.beta_c[e]] = P.beta_v[e];
+    }
+    std::vector<int> lam_slot(P.lam_c.size());
+    for (size_t e = 0; e < P.lam_c.size(); ++e) {
+        lam_slot[e] = P.win_slot(P.lam_c[e]);
+        if (lam_slot[e] < 0) return fail(SB_UNSUPPORTED, "internal: lambda column outside window");
+    }
+    std::vector<double> dscale(k);
+    for (int d = 0; d < k; ++d) dscale[d] = P.rowscale[P.drow[d]];
+
+    Packer pk;
+    size_t o_fwd[2], o_bwd[2], o_beta[2], o_lamv[2], o_dlu[2], o_ds[2];
+    o_fwd[0] = pk.addv(fwd);
+    o_bwd[0] = pk.addv(bwd);
+    o_beta[0] = pk.addv(betaW);
+    o_lamv[0] = pk.addv(P.lam_v);
+    o_dlu[0] = pk.addv(P.dlu);
+    o_ds[0] = pk.addv(dscale);
+    o_fwd[1] = pk.addv(conv<float>(fwd));
+    o_bwd[1] = pk.addv(conv<float>(bwd));
+    o_beta[1] = pk.addv(conv<float>(betaW));
+    o_lamv[1] = pk.addv(conv<float>(P.lam_v));
+    o_dlu[1] = pk.addv(conv<float>(P.dlu));
+    o_ds[1] = pk.addv(conv<float>(dscale));
+    size_t o_lamr = pk.addv(P.lam_r), o_lams = pk.addv(lam_slot), o_dpiv = pk.addv(P.dpiv), o_drow = pk.addv(P.drow);
+    h->blob_bytes = std::max<size_t>(pk.bytes.size(), 16);
+    cudaError_t e = cudaMalloc(&h->blob, h->blob_bytes);
+    if (e != cudaSuccess) return fail(SB_NOMEM, std::string("cudaMalloc(blob): ") + cudaGetErrorString(e));
+    e = cudaMemcpy(h->blob, pk.bytes.data(), pk.bytes.size(), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return fail(SB_CUDA, std::string("cudaMemcpy(blob): ") + cudaGetErrorString(e));
+    auto at = [&](size_t off) { return (const void *)((const unsigned char *)h->blob + off); };
+    sb::DevPlan &d = h->dp;
+    d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K;
+    d.S = P.S; d.seg_base = P.seg_base; d.seg_rem = P.seg_rem;
+    d.carry_f = P.carry_f; d.carry_b = P.carry_b;
+    d.Wh = P.Wh; d.Wt = P.Wt; d.nlam = (int)P.lam_v.size();
+    d.fstride = FS; d.bstride = BS;
+    for (int c = 0; c < 2; ++c) {
+        d.fwd[c] = at(o_fwd[c]); d.bwd[c] = at(o_bwd[c]); d.betaW[c] = at(o_beta[c]);
+        d.lam_v[c] = at(o_lamv[c]); d.dlu[c] = at(o_dlu[c]); d.dscale[c] = at(o_ds[c]);
+    }
+    d.lam_r = (const int *)at(o_lamr); d.lam_slot = (const int *)at(o_lams);
+    d.dpiv = (const int *)at(o_dpiv); d.drow = (const int *)at(o_drow);
+    return 0;
+}
+
+int do_solve(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t bstride, int64_t pstride,
+             cudaStream_t stream) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (h->host_only) return fail(SB_UNSUPPORTED, "handle was created with SB_FLAG_HOST_ONLY");
+    if (dtype != SB_F64 && dtype != SB_F32) return fail(SB_INVALID_ARG, "dtype must be SB_F64 or SB_F32");
+    if (batch < 0) return fail(SB_INVALID_ARG, "batch < 0");
+    if (batch == 0) return SB_OK;
+    if (!rhs) return fail(SB_INVALID_ARG, "rhs is NULL");
+    if (bstride <= 0 || pstride <= 0) return fail(SB_INVALID_ARG, "strides must be positive");
+    const int64_t n = h->plan.n;
+    // one-to-one map (j, r) -> r*bstride + j*pstride for the two supported families
+    bool ok = (bstride == 1 && pstride >= batch) || (pstride == 1 && bstride >= n) ||
+              (bstride >= pstride * n) || (pstride >= bstride * batch);
+    if (!ok) return fail(SB_INVALID_ARG, "strides alias: (row, rhs) -> offset is not one-to-one");
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != h->device) cudaSetDevice(h->device);
+    sb::SolveArgs a{rhs, batch, bstride, pstride, dtype, stream};
+    char err[256] = {0};
+    int st = sb::launch_solve(h->dp, a, h->num_sms, err, sizeof(err));
+    if (cur != h->device) cudaSetDevice(cur);
+    if (st) return fail(st, err);
+    return SB_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, const double *knots, int split_lo,
+                                          int split_hi, int flags) {
+    spline_builder *h = new (std::nothrow) spline_builder();
+    if (!h) { fail(SB_NOMEM, "out of host memory"); return nullptr; }
+    try {
+        sb::Status st = sb::build_plan(h->plan, degree, n_points, bc, knots, split_lo, split_hi, LMAX_SEG);
+        if (st.code) { fail(st.code, st.msg); delete h; return nullptr; }
+    } catch (const std::bad_alloc &) {
+        fail(SB_NOMEM, "out of host memory in create"); delete h; return nullptr;
+    } catch (...) {
+        fail(SB_INVALID_ARG, "unexpected failure in create"); delete h; return nullptr;
+    }
+    h->host_only = (flags & SB_FLAG_HOST_ONLY) != 0;
+    if (!h->host_only) {
+        if (cudaGetDevice(&h->device) != cudaSuccess) { fail(SB_CUDA, "no CUDA device"); delete h; return nullptr; }
+        cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device);
+        if (upload(h)) { spline_builder_destroy(h); return nullptr; }
+    }
+    return h;
+}
+
+spline_builder_t spline_builder_create(int degree, int n_points, int bc, const double *knots) {
+    return spline_builder_create_ex(degree, n_points, bc, knots, -1, -1, 0);
+}
+
+int spline_builder_solve(spline_builder_t h, double *rhs, int64_t batch, int64_t batch_stride, void *stream) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (batch_stride == 1) return do_solve(h, rhs, SB_F64, batch, 1, batch, (cudaStream_t)stream);
+    if (batch_stride >= h->plan.n) return do_solve(h, rhs, SB_F64, batch, batch_stride, 1, (cudaStream_t)stream);
+    return fail(SB_INVALID_ARG, "batch_stride must be 1 or >= n (use spline_builder_solve_strided)");
+}
+
+int spline_builder_solve_f32(spline_builder_t h, float *rhs, int64_t batch, int64_t batch_stride, void *stream) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (batch_stride == 1) return do_solve(h, rhs, SB_F32, batch, 1, batch, (cudaStream_t)stream);
+    if (batch_stride >= h->plan.n) return do_solve(h, rhs, SB_F32, batch, batch_stride, 1, (cudaStream_t)stream);
+    return fail(SB_INVALID_ARG, "batch_stride must be 1 or >= n (use spline_builder_solve_strided)");
+}
+
+int spline_builder_solve_strided(spline_builder_t h, void *rhs, int dtype, int64_t batch, int64_t batch_stride,
+                                 int64_t point_stride, void *stream) {
+    return do_solve(h, rhs, dtype, batch, batch_stride, point_stride, (cudaStream_t)stream);
+}
+
+int spline_builder_solve_host(spline_builder_t h, void *host_rhs, int dtype, int64_t batch, int64_t ld) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (h->host_only) return fail(SB_UNSUPPORTED, "handle was created with SB_FLAG_HOST_ONLY");
+    if (dtype != SB_F64 && dtype != SB_F32) return fail(SB_INVALID_ARG, "dtype must be SB_F64 or SB_F32");
+    if (batch < 0 || ld < batch) return fail(SB_INVALID_ARG, "need 0 <= batch <= ld");
+    if (batch == 0) return SB_OK;
+    if (!host_rhs) return fail(SB_INVALID_ARG, "host_rhs is NULL");
+    std::lock_guard<std::mutex> lock(h->host_mu);
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != h->device) cudaSetDevice(h->device);
+    const size_t esz = dtype == SB_F64 ? 8 : 4;
+    const int64_t n = h->plan.n;
+    // chunk of RHS per pipeline stage: ~64 MB, multiple of 16 columns
+    int64_t chunk = std::max<int64_t>(16, ((int64_t)(64ll << 20) / (n * (int64_t)esz)) / 16 * 16);
+    chunk = std::min<int64_t>(chunk, (batch + 15) / 16 * 16);
+    const size_t need = (size_t)chunk * n * esz;
+    int rc = SB_OK;
+    if (need > h->stage_bytes) {
+        for (int i = 0; i < 3; ++i) { if (h->stage[i]) cudaFree(h->stage[i]); h->stage[i] = nullptr; }
+        h->stage_bytes = 0;
+        for (int i = 0; i < 3; ++i)
+            if (cudaMalloc(&h->stage[i], need) != cudaSuccess) rc = fail(SB_NOMEM, "cudaMalloc(staging) failed");
+        if (rc) {
+            for (int i = 0; i < 3; ++i) { if (h->stage[i]) cudaFree(h->stage[i]); h->stage[i] = nullptr; }
+        } else {
+            h->stage_bytes = need;
+        }
+    }
+    for (int i = 0; i < 3 && !rc; ++i)
+        if (!h->streams[i] && cudaStreamCreateWithFlags(&h->streams[i], cudaStreamNonBlocking) != cudaSuccess)
+            rc = fail(SB_CUDA, "cudaStreamCreate failed");
+    unsigned char *host = static_cast<unsigned char *>(host_rhs);
+    for (int64_t c0 = 0, it = 0; c0 < batch && !rc; c0 += chunk, ++it) {
+        const int64_t w = std::min<int64_t>(chunk, batch - c0);
+        const int si = (int)(it % 3);
+        cudaStream_t st = h->streams[si];
+        void *dbuf = h->stage[si];
+        cudaError_t e = cudaMemcpy2DAsync(dbuf, w * esz, host + c0 * esz, ld * esz, w * esz, n,
+                                          cudaMemcpyHostToDevice, st);
+        if (e != cudaSuccess) { rc = fail(SB_CUDA, std::string("H2D: ") + cudaGetErrorString(e)); break; }
+        int s = do_solve(h, dbuf, dtype, w, 1, w, st);
+        if (s) { rc = s; break; }
+        e = cudaMemcpy2DAsync(host + c0 * esz, ld * esz, dbuf, w * esz, w * esz, n, cudaMemcpyDeviceToHost, st);
+        if (e != cudaSuccess) { rc = fail(SB_CUDA, std::string("D2H: ") + cudaGetErrorString(e)); break; }
+    }
+    for (int i = 0; i < 3; ++i)
+        if (h->streams[i]) {
+            cudaError_t e = cudaStreamSynchronize(h->streams[i]);
+            if (e != cudaSuccess && !rc) rc = fail(SB_CUDA, std::string("solve_host: ") + cudaGetErrorString(e));
+        }
+    if (cur != h->device) cudaSetDevice(cur);
+    return rc;
+}
+
+void spline_builder_destroy(spline_builder_t h) {
+    if (!h) return;
+    if (!h->host_only) {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (h->device >= 0 && cur != h->device) cudaSetDevice(h->device);
+        if (h->blob) cudaFree(h->blob);
+        for (int i = 0; i < 3; ++i) {
+            if (h->stage[i]) cudaFree(h->stage[i]);
+            if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
+        }
+        if (h->device >= 0 && cur != h->device) cudaSetDevice(cur);
+    }
+    delete h;
+}
+
+int spline_builder_get_info(spline_builder_t h, spline_builder_info_t *info) {
+    if (!h || !info) return fail(SB_INVALID_ARG, "null argument");
+    const sb::Plan &P = h->plan;
+    info->degree = P.p; info->bc = P.bc; info->n_cells = P.N; info->nbasis = P.n;
+    info->split_lo = P.s_lo; info->split_hi = P.s_hi; info->k = P.k;
+    info->q_kl = P.kl; info->q_ku = P.ku; info->q_type = P.qtype;
+    info->nnz_lambda = (int)P.lam_v.size(); info->nnz_beta = (int)P.beta_v.size();
+    int head = 0, tail = 0;
+    for (int r : P.beta_r) { if (r < P.Wh) head = std::max(head, r + 1); else tail = std::max(tail, P.nQ - r); }
+    info->beta_rows_head = head; info->beta_rows_tail = tail;
+    info->n_segments = P.S; info->seg_len = P.Lseg;
+    info->carry_fwd = P.carry_f; info->carry_bwd = P.carry_b;
+    info->max_pivot_growth = P.growth;
+    return SB_OK;
+}
+
+int64_t spline_builder_nbasis(spline_builder_t h) { return h ? h->plan.n : -1; }
+
+int spline_builder_get_blocks(spline_builder_t h, int *lam_rows, int *lam_cols, double *lam_vals, int *beta_rows,
+                              int *beta_cols, double *beta_vals, double *delta_prime) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    const sb::Plan &P = h->plan;
+    for (size_t e = 0; e < P.lam_v.size(); ++e) {
+        if (lam_rows) lam_rows[e] = P.lam_r[e];
+        if (lam_cols) lam_cols[e] = P.lam_c[e];
+        if (lam_vals) lam_vals[e] = P.lam_v[e];
+    }
+    for (size_t e = 0; e < P.beta_v.size(); ++e) {
+        if (beta_rows) beta_rows[e] = P.beta_r[e];
+        if (beta_cols) beta_cols[e] = P.beta_c[e];
+        if (beta_vals) beta_vals[e] = P.beta_v[e];
+    }
+    if (delta_prime && !P.dprime.empty()) std::memcpy(delta_prime, P.dprime.data(), P.dprime.size() * sizeof(double));
+    return SB_OK;
+}
+
+int spline_builder_solve_cpu_plan(spline_builder_t h, double *rhs, int64_t batch, int64_t batch_stride,
+                                  int64_t point_stride) {
+    if (!h || !rhs || batch < 0) return fail(SB_INVALID_ARG, "bad argument");
+    sb::plan_solve_cpu(h->plan, rhs, batch, batch_stride, point_stride);
+    return SB_OK;
+}
+
+const char *spline_builder_last_error(void) { return g_err.c_str(); }
+int spline_builder_last_status(void) { return g_status; }
+const char *spline_builder_version(void) { return "b200-spline-build 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -1,0 +1,572 @@
+// plan.cpp -- host create step (see plan.hpp).
+//
+// Collocation matrix: span-based de Boor triangular scheme (BSPLVB) and its
+// derivative extension, evaluated in local (cell-relative) coordinates: every
+// knot difference is a sum of cell widths and every point is (span, offset).
+// Schur split / factorisation / corners: PAPER.md Eq. 3-6, Table I
+// (P:95-101), COO corners (Listing 5-6).
+#include "plan.hpp"
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <map>
+#include <random>
+
+namespace sb {
+namespace {
+
+long lmod(long a, long m) {
+    long r = a % m;
+    return r < 0 ? r + m : r;
+}
+
+struct Space {
+    int p, bc, N, n, nbc;
+    const double *h;
+
+    double width(long g) const {
+        if (bc == PERIODIC) return h[lmod(g, N)];
+        return (g >= p && g < N + p) ? h[g - p] : 0.0;
+    }
+    // t_a - t_b (a >= b) as a sum of interval widths
+    double kd(long a, long b) const {
+        double s = 0.0;
+        for (long g = b; g < a; ++g) s += width(g);
+        return s;
+    }
+    long first_knot(int j) const { return bc == PERIODIC ? j - (p + 1) / 2 : j; }
+    int basis_of(long q) const { return bc == PERIODIC ? (int)lmod(q + (p + 1) / 2, N) : (int)q; }
+    long span_of_cell(int c) const { return bc == PERIODIC ? c : (long)c + p; }
+};
+
+struct RowPt {
+    long span;  // knot interval index containing the point
+    double u;   // offset from t_span
+    int deriv;
+};
+
+// BSPLVB (de Boor): values of the q+1 degree-q B-splines with first knots
+// span-q .. span at x = t_span + u.
+void bsplvb(const Space &S, long mu, double u, int q, double *b) {
+    double dl[16], dr[16];
+    b[0] = 1.0;
+    for (int j = 0; j < q; ++j) {
+        dr[j] = S.kd(mu + 1 + j, mu) - u;
+        dl[j] = u + S.kd(mu, mu - j);
+        double saved = 0.0;
+        for (int r = 0; r <= j; ++r) {
+            double den = dr[r] + dl[j - r];
+            double term = den > 0.0 ? b[r] / den : 0.0;
+            b[r] = saved + dr[r] * term;
+            saved = dl[j - r] * term;
+        }
+        b[j + 1] = saved;
+    }
+}
+
+// d-th derivative of the p+1 degree-p B-splines with first knots span-p..span:
+// values of degree p-d, then d applications of
+//   D B_{i,q} = q (B_{i,q-1}/(t_{i+q}-t_i) - B_{i+1,q-1}/(t_{i+q+1}-t_{i+1})).
+void bsplvd(const Space &S, long mu, double u, int d, double *out) {
+    const int p = S.p;
+    double v[16], w[16];
+    bsplvb(S, mu, u, p - d, v);
+    for (int q = p - d + 1; q <= p; ++q) {
+        for (int r = 0; r <= q; ++r) {
+            long i = mu - q + r;
+            double acc = 0.0;
+            if (r - 1 >= 0) {
+                double den = S.kd(i + q, i);
+                if (den > 0.0) acc += v[r - 1] / den;
+            }
+            if (r <= q - 1) {
+                double den = S.kd(i + q + 1, i + 1);
+                if (den > 0.0) acc -= v[r] / den;
+            }
+            w[r] = q * acc;
+        }
+        for (int r = 0; r <= q; ++r) v[r] = w[r];
+    }
+    for (int r = 0; r <= p; ++r) out[r] = v[r];
+}
+
+// Greville abscissa (t_{q+1}+...+t_{q+p})/p of the basis with first knot q,
+// located as (span, u); the closed right end of the last interval is kept.
+RowPt greville(const Space &S, int j) {
+    long q = S.first_knot(j);
+    double off = 0.0;
+    for (int l = 1; l <= S.p; ++l) off += S.kd(q + l, q);
+    off /= S.p;
+    long last = -1;
+    double lastlo = 0.0;
+    for (int l = 0; l <= S.p; ++l) {
+        long g = q + l;
+        double w = S.width(g);
+        if (w <= 0.0) continue;
+        double lo = S.kd(g, q);
+        last = g;
+        lastlo = lo;
+        if (off >= lo && off < lo + w) return RowPt{g, off - lo, 0};
+    }
+    return RowPt{last, off - lastlo, 0};
+}
+
+double dmax_abs(const std::vector<double> &v) {
+    double m = 0.0;
+    for (double x : v) m = std::max(m, std::fabs(x));
+    return m;
+}
+
+struct SplitResult {
+    int code = 0;
+    std::string msg;
+};
+
+// try one Schur split; fills P on success
+SplitResult try_split(Plan &P, int slo, int shi) {
+    SplitResult R;
+    const int n = P.n;
+    const int k = slo + shi;
+    if (slo < 0 || shi < 0 || k > KMAX_DELTA || k > n) return {1, "split out of range"};
+    const int nQ = n - k;
+    // every equilibrated (scaled) row must be a delta row (kernel reads Q rows unscaled)
+    for (int i = slo; i < n - shi; ++i)
+        if (P.rowscale[i] != 1.0) return {1, "scaled (Hermite derivative) row inside Q"};
+    auto dindex = [&](int g) { return g < slo ? g : (g >= n - shi ? slo + (g - (n - shi)) : -1); };
+    // Q band
+    int kl = 0, ku = 0;
+    for (int i = 0; i < nQ; ++i) {
+        const SparseRow &row = P.A[slo + i];
+        for (size_t e = 0; e < row.col.size(); ++e) {
+            int c = row.col[e];
+            if (c < slo || c >= n - shi || row.val[e] == 0.0) continue;
+            int o = (c - slo) - i;
+            kl = std::max(kl, -o);
+            ku = std::max(ku, o);
+        }
+    }
+    if (kl > KMAX_BAND || ku > KMAX_BAND) return {5, "Q band too wide"};
+    const int K = std::max(1, std::max(kl, ku));
+    // dense band of Q: Qb[i*(2K+1) + (o+K)]
+    const int BW = 2 * K + 1;
+    std::vector<double> Qb((size_t)nQ * BW, 0.0);
+    std::vector<double> gam((size_t)nQ * k, 0.0), lam((size_t)k * nQ, 0.0), del((size_t)k * k, 0.0);
+    for (int g = 0; g < n; ++g) {
+        const SparseRow &row = P.A[g];
+        int dg = dindex(g);
+        for (size_t e = 0; e < row.col.size(); ++e) {
+            int c = row.col[e];
+            double v = row.val[e];
+            int dc = dindex(c);
+            if (dg < 0 && dc < 0) Qb[(size_t)(g - slo) * BW + ((c - slo) - (g - slo) + K)] += v;
+            else if (dg < 0) gam[(size_t)(g - slo) * k + dc] += v;
+            else if (dc < 0) lam[(size_t)dg * nQ + (c - slo)] += v;
+            else del[(size_t)dg * k + dc] += v;
+        }
+    }
+    auto Q = [&](int i, int j) -> double & { return Qb[(size_t)i * BW + (j - i + K)]; };
+    const double qmax = dmax_abs(Qb);
+    std::vector<double> Lb((size_t)nQ * K, 0.0), Ub((size_t)nQ * K, 0.0), dinv(nQ, 0.0);
+    int qtype = Q_GBTRS;
+    double growth = 1.0;
+    bool done = false;
+    if (nQ > 0) {
+        // symmetric?  (PAPER Table I: uniform -> PDS)
+        bool sym = true;
+        for (int i = 0; i < nQ && sym; ++i)
+            for (int m = 1; m <= K && i + m < nQ; ++m)
+                if (std::fabs(Q(i, i + m) - Q(i + m, i)) > 4e-16 * qmax) { sym = false; break; }
+        if (sym) {
+            // banded LDL^T (pttrf for K=1, pbtrf-equivalent otherwise), no pivoting
+            std::vector<double> L((size_t)nQ * K, 0.0), d(nQ, 0.0);  // L[i*K+m-1] = L(i,i-m)
+            bool pd = true;
+            for (int j = 0; j < nQ && pd; ++j) {
+                double dj = Q(j, j);
+                for (int m = 1; m <= K && j - m >= 0; ++m) dj -= L[(size_t)j * K + m - 1] * L[(size_t)j * K + m - 1] * d[j - m];
+                if (!(dj > 0.0)) { pd = false; break; }
+                d[j] = dj;
+                for (int i = j + 1; i <= j + K && i < nQ; ++i) {
+                    double v = Q(i, j);
+                    // sum over c < j inside both bands: L(i,c) L(j,c) d_c
+                    for (int c = std::max(0, i - K); c < j; ++c) {
+                        if (j - c > K) continue;
+                        v -= L[(size_t)i * K + (i - c) - 1] * L[(size_t)j * K + (j - c) - 1] * d[c];
+                    }
+                    L[(size_t)i * K + (i - j) - 1] = v / dj;
+                }
+            }
+            if (pd) {
+                for (int i = 0; i < nQ; ++i) {
+                    dinv[i] = 1.0 / d[i];
+                    for (int m = 1; m <= K; ++m) {
+                        Lb[(size_t)i * K + m - 1] = L[(size_t)i * K + m - 1];
+                        Ub[(size_t)i * K + m - 1] = (i + m < nQ) ? L[(size_t)(i + m) * K + m - 1] : 0.0;
+                    }
+                }
+                qtype = (K == 1) ? Q_PTTRS : Q_PBTRS;
+                growth = 1.0;
+                done = true;
+            }
+        }
+        if (!done) {
+            // banded LU without row interchanges (gbtrf path).  Accepted only if
+            // it is stable here (collocation matrices are totally positive, so
+            // elimination without pivoting is stable; R5).
+            std::vector<double> W = Qb;
+            auto Wa = [&](int i, int j) -> double & { return W[(size_t)i * BW + (j - i + K)]; };
+            double lmax = 0.0, umax = 0.0;
+            for (int j = 0; j < nQ; ++j) {
+                double piv = Wa(j, j);
+                if (!(std::fabs(piv) > 1e-13 * qmax)) return {2, "zero pivot in Q"};
+                for (int i = j + 1; i <= std::min(nQ - 1, j + kl); ++i) {
+                    double l = Wa(i, j) / piv;
+                    Wa(i, j) = l;
+                    lmax = std::max(lmax, std::fabs(l));
+                    if (l != 0.0)
+                        for (int c = j + 1; c <= std::min(nQ - 1, j + ku); ++c) Wa(i, c) -= l * Wa(j, c);
+                }
+            }
+            for (int i = 0; i < nQ; ++i)
+                for (int c = i; c <= std::min(nQ - 1, i + ku); ++c) umax = std::max(umax, std::fabs(Wa(i, c)));
+            growth = umax / qmax;
+            if (lmax > 1e3 || growth > 1e3) return {2, "no-pivot LU of Q unstable"};
+            for (int i = 0; i < nQ; ++i) {
+                double u = Wa(i, i);
+                dinv[i] = 1.0 / u;
+                for (int m = 1; m <= K; ++m) {
+                    Lb[(size_t)i * K + m - 1] = (i - m >= 0 && m <= kl) ? Wa(i, i - m) : 0.0;
+                    Ub[(size_t)i * K + m - 1] = (i + m < nQ && m <= ku) ? Wa(i, i + m) / u : 0.0;
+                }
+            }
+            qtype = Q_GBTRS;
+        }
+    }
+    // beta = Q^{-1} gamma (Eq. 4), one banded solve per delta column
+    std::vector<double> beta((size_t)nQ * k, 0.0), v(nQ);
+    for (int c = 0; c < k; ++c) {
+        for (int i = 0; i < nQ; ++i) v[i] = gam[(size_t)i * k + c];
+        for (int i = 0; i < nQ; ++i)
+            for (int m = 1; m <= K && i - m >= 0; ++m) v[i] -= Lb[(size_t)i * K + m - 1] * v[i - m];
+        for (int i = nQ - 1; i >= 0; --i) {
+            double acc = v[i] * dinv[i];
+            for (int m = 1; m <= K && i + m < nQ; ++m) acc -= Ub[(size_t)i * K + m - 1] * v[i + m];
+            v[i] = acc;
+        }
+        for (int i = 0; i < nQ; ++i) beta[(size_t)i * k + c] = v[i];
+    }
+    // delta' = delta - lambda beta (Eq. 4)
+    std::vector<double> dp = del;
+    for (int r = 0; r < k; ++r)
+        for (int c = 0; c < k; ++c) {
+            double acc = 0.0;
+            for (int i = 0; i < nQ; ++i) acc += lam[(size_t)r * nQ + i] * beta[(size_t)i * k + c];
+            dp[(size_t)r * k + c] -= acc;
+        }
+    // getrf(delta') with partial pivoting (first max, like idamax)
+    std::vector<double> lu = dp;
+    std::vector<int> piv(k);
+    double dmax = dmax_abs(dp);
+    for (int j = 0; j < k; ++j) {
+        int pr = j;
+        double best = std::fabs(lu[(size_t)j * k + j]);
+        for (int i = j + 1; i < k; ++i)
+            if (std::fabs(lu[(size_t)i * k + j]) > best) { best = std::fabs(lu[(size_t)i * k + j]); pr = i; }
+        piv[j] = pr;
+        if (!(best > 1e-13 * dmax)) return {2, "delta' singular"};
+        if (pr != j)
+            for (int c = 0; c < k; ++c) std::swap(lu[(size_t)j * k + c], lu[(size_t)pr * k + c]);
+        for (int i = j + 1; i < k; ++i) {
+            double l = lu[(size_t)i * k + j] / lu[(size_t)j * k + j];
+            lu[(size_t)i * k + j] = l;
+            for (int c = j + 1; c < k; ++c) lu[(size_t)i * k + c] -= l * lu[(size_t)j * k + c];
+        }
+    }
+    // commit
+    P.s_lo = slo; P.s_hi = shi; P.k = k; P.nQ = nQ;
+    P.drow.resize(k);
+    for (int d = 0; d < k; ++d) P.drow[d] = d < slo ? d : n - shi + (d - slo);
+    P.kl = kl; P.ku = ku; P.K = K; P.qtype = qtype; P.growth = growth;
+    P.Lb.swap(Lb); P.Ub.swap(Ub); P.dinv.swap(dinv);
+    P.beta_full.swap(beta);
+    P.dprime = dp; P.dlu.swap(lu); P.dpiv.swap(piv);
+    P.lam_r.clear(); P.lam_c.clear(); P.lam_v.clear();
+    for (int r = 0; r < k; ++r)
+        for (int i = 0; i < nQ; ++i)
+            if (lam[(size_t)r * nQ + i] != 0.0) {
+                P.lam_r.push_back(r); P.lam_c.push_back(i); P.lam_v.push_back(lam[(size_t)r * nQ + i]);
+            }
+    P.beta_r.clear(); P.beta_c.clear(); P.beta_v.clear();
+    for (int i = 0; i < nQ; ++i)
+        for (int c = 0; c < k; ++c) {
+            double b = P.beta_full[(size_t)i * k + c];
+            if (std::fabs(b) > BETA_DROP) { P.beta_r.push_back(i); P.beta_c.push_back(c); P.beta_v.push_back(b); }
+        }
+    return R;
+}
+
+// segment partition + spike vectors + carry depths + windows
+void build_segments(Plan &P, int Lmax) {
+    const int nQ = P.nQ, K = P.K;
+    P.Lmax = Lmax;
+    int S = nQ > 0 ? (nQ + Lmax - 1) / Lmax : 1;
+    if (S > 1 && nQ / S < K) S = 1;
+    P.S = S;
+    P.seg_base = nQ / S;
+    P.seg_rem = nQ % S;
+    P.Lseg = P.seg_base + (P.seg_rem ? 1 : 0);
+    P.gspk.assign((size_t)nQ * K, 0.0);
+    P.hspk.assign((size_t)nQ * K, 0.0);
+    std::vector<double> y(nQ + 2 * K);
+    for (int s = 1; s < S; ++s) {
+        int a = P.seg_start(s), len = P.seg_len(s);
+        for (int m = 1; m <= K; ++m) {
+            // y indices shifted by K: y[K + i] = y_{a+i}, y[K - m'] = inflow state
+            std::fill(y.begin(), y.begin() + K + len, 0.0);
+            y[K - m] = 1.0;
+            for (int i = 0; i < len; ++i) {
+                int row = a + i;
+                double acc = 0.0;
+                for (int mm = 1; mm <= K; ++mm) acc -= P.Lb[(size_t)row * K + mm - 1] * y[K + i - mm];
+                y[K + i] = acc;
+                P.gspk[(size_t)row * K + m - 1] = acc;
+            }
+        }
+    }
+    for (int s = 0; s + 1 < S; ++s) {
+        int a = P.seg_start(s), len = P.seg_len(s);
+        for (int m = 1; m <= K; ++m) {
+            // x[i] = x_{a+i}, i in [0, len+K)
+            std::fill(y.begin(), y.begin() + len + K, 0.0);
+            y[len + m - 1] = 1.0;
+            for (int i = len - 1; i >= 0; --i) {
+                int row = a + i;
+                double acc = 0.0;
+                for (int mm = 1; mm <= K; ++mm) acc -= P.Ub[(size_t)row * K + mm - 1] * y[i + mm];
+                y[i] = acc;
+                P.hspk[(size_t)row * K + m - 1] = acc;
+            }
+        }
+    }
+    // carry depths: smallest T with prod ||G|| <= 2^-60 or reaching an exact end
+    const double eps = std::ldexp(1.0, -60);
+    auto Gnorm = [&](int t) {  // forward transfer of segment t (rows at its end)
+        int end = P.seg_start(t) + P.seg_len(t);
+        double nrm = 0.0;
+        for (int j = 0; j < K; ++j) {
+            double s = 0.0;
+            for (int m = 0; m < K; ++m) s += std::fabs(P.gspk[(size_t)(end - 1 - j) * K + m]);
+            nrm = std::max(nrm, s);
+        }
+        return nrm;
+    };
+    auto Hnorm = [&](int t) {
+        int a = P.seg_start(t);
+        double nrm = 0.0;
+        for (int j = 0; j < K; ++j) {
+            double s = 0.0;
+            for (int m = 0; m < K; ++m) s += std::fabs(P.hspk[(size_t)(a + j) * K + m]);
+            nrm = std::max(nrm, s);
+        }
+        return nrm;
+    };
+    P.carry_f = 0;
+    for (int s = 1; s < S; ++s) {
+        int T = 0;
+        double prod = 1.0;
+        while (true) {
+            ++T;
+            int t = s - T;
+            if (t == 0) break;
+            prod *= Gnorm(t);
+            if (prod <= eps) break;
+        }
+        P.carry_f = std::max(P.carry_f, T);
+    }
+    P.carry_b = 0;
+    for (int s = 0; s + 1 < S; ++s) {
+        int T = 0;
+        double prod = 1.0;
+        while (true) {
+            ++T;
+            int t = s + T;
+            if (t == S - 1) break;
+            prod *= Hnorm(t);
+            if (prod <= eps) break;
+        }
+        P.carry_b = std::max(P.carry_b, T);
+    }
+    // windows: every lambda column and beta row
+    int head = -1, tail = nQ;
+    auto note = [&](int q) {
+        if (q < nQ / 2 + 1) head = std::max(head, q);
+        else tail = std::min(tail, q);
+    };
+    for (int c : P.lam_c) note(c);
+    for (int r : P.beta_r) note(r);
+    P.Wh = head + 1;
+    P.Wt = nQ - tail;
+    if (P.Wh + P.Wt >= nQ) { P.Wh = nQ; P.Wt = 0; }
+}
+
+}  // namespace
+
+void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, int64_t pstride) {
+    const int n = P.n, nQ = P.nQ, k = P.k, K = P.K;
+    std::vector<double> v(nQ), x1(k);
+    for (int64_t r = 0; r < batch; ++r) {
+        double *col = rhs + r * bstride;
+        for (int i = 0; i < nQ; ++i) v[i] = col[(int64_t)(P.s_lo + i) * pstride];
+        for (int d = 0; d < k; ++d) x1[d] = col[(int64_t)P.drow[d] * pstride] * P.rowscale[P.drow[d]];
+        // step 2: Q x0' = b0
+        for (int i = 0; i < nQ; ++i)
+            for (int m = 1; m <= K && i - m >= 0; ++m) v[i] -= P.Lb[(size_t)i * K + m - 1] * v[i - m];
+        for (int i = nQ - 1; i >= 0; --i) {
+            double acc = v[i] * P.dinv[i];
+            for (int m = 1; m <= K && i + m < nQ; ++m) acc -= P.Ub[(size_t)i * K + m - 1] * v[i + m];
+            v[i] = acc;
+        }
+        // step 3: delta' x1 = b1 - lambda x0'
+        for (size_t e = 0; e < P.lam_v.size(); ++e) x1[P.lam_r[e]] -= P.lam_v[e] * v[P.lam_c[e]];
+        for (int d = 0; d < k; ++d)
+            if (P.dpiv[d] != d) std::swap(x1[d], x1[P.dpiv[d]]);
+        for (int i = 1; i < k; ++i)
+            for (int j = 0; j < i; ++j) x1[i] -= P.dlu[(size_t)i * k + j] * x1[j];
+        for (int i = k - 1; i >= 0; --i) {
+            for (int j = i + 1; j < k; ++j) x1[i] -= P.dlu[(size_t)i * k + j] * x1[j];
+            x1[i] /= P.dlu[(size_t)i * k + i];
+        }
+        // step 4: x0 = x0' - beta x1
+        for (size_t e = 0; e < P.beta_v.size(); ++e) v[P.beta_r[e]] -= P.beta_v[e] * x1[P.beta_c[e]];
+        for (int i = 0; i < nQ; ++i) col[(int64_t)(P.s_lo + i) * pstride] = v[i];
+        for (int d = 0; d < k; ++d) col[(int64_t)P.drow[d] * pstride] = x1[d];
+    }
+}
+
+Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi,
+                  int Lmax) {
+    P = Plan();
+    if (degree < 1 || degree > 5) return {1, "degree must be in 1..5"};
+    if (bc != PERIODIC && bc != GREVILLE && bc != HERMITE) return {1, "unknown boundary condition"};
+    P.p = degree;
+    P.bc = bc;
+    if (bc == PERIODIC) { P.N = n_points; P.n = P.N; }
+    else if (bc == GREVILLE) { P.N = n_points - degree; P.n = P.N + degree; }
+    else {
+        P.N = (degree % 2) ? n_points - 1 : n_points;
+        P.nbc = (degree % 2) ? (degree - 1) / 2 : degree / 2;
+        P.n = P.N + degree;
+    }
+    if (P.N < 1) return {1, "too few points for this degree / boundary condition"};
+    if (bc == PERIODIC && P.N < 2) return {1, "periodic spline needs at least 2 cells"};
+    const int N = P.N, n = P.n, p = P.p;
+    P.h.resize(N);
+    for (int c = 0; c < N; ++c) {
+        P.h[c] = knots ? knots[c + 1] - knots[c] : 1.0 / (double)N;  // uniform: exact equal widths (R1)
+        if (!(P.h[c] > 0.0) || !std::isfinite(P.h[c])) return {1, "breakpoints must be strictly increasing"};
+    }
+    Space S{p, bc, N, n, P.nbc, P.h.data()};
+    // rows
+    std::vector<RowPt> rows(n);
+    P.rowscale.assign(n, 1.0);
+    if (bc != HERMITE) {
+        for (int j = 0; j < n; ++j) rows[j] = greville(S, j);
+    } else {
+        int r = 0;
+        for (int d = 1; d <= P.nbc; ++d) { rows[r] = RowPt{S.span_of_cell(0), 0.0, d}; P.rowscale[r] = std::pow(P.h[0], d); ++r; }
+        if (p % 2) {
+            for (int i = 0; i <= N; ++i) {
+                rows[r] = i < N ? RowPt{S.span_of_cell(i), 0.0, 0} : RowPt{S.span_of_cell(N - 1), P.h[N - 1], 0};
+                ++r;
+            }
+        } else {
+            for (int c = 0; c < N; ++c) { rows[r] = RowPt{S.span_of_cell(c), 0.5 * P.h[c], 0}; ++r; }
+        }
+        for (int d = 1; d <= P.nbc; ++d) {
+            rows[r] = RowPt{S.span_of_cell(N - 1), P.h[N - 1], d};
+            P.rowscale[r] = std::pow(P.h[N - 1], d);
+            ++r;
+        }
+    }
+    // equilibrated sparse rows: rowscale * (d^deriv B_j)(point)
+    P.A.assign(n, SparseRow());
+    for (int i = 0; i < n; ++i) {
+        double vals[16];
+        if (rows[i].deriv == 0) bsplvb(S, rows[i].span, rows[i].u, p, vals);
+        else bsplvd(S, rows[i].span, rows[i].u, rows[i].deriv, vals);
+        std::map<int, double> acc;
+        for (int r = 0; r <= p; ++r) acc[S.basis_of(rows[i].span - p + r)] += vals[r] * P.rowscale[i];
+        for (auto &kv : acc)
+            if (kv.second != 0.0) { P.A[i].col.push_back(kv.first); P.A[i].val.push_back(kv.second); }
+        if (P.A[i].col.empty()) return {2, "empty collocation row"};
+    }
+    // candidate splits
+    std::vector<std::pair<int, int>> cands;
+    if (split_lo >= 0 || split_hi >= 0) {
+        if (split_lo < 0 || split_hi < 0) return {1, "give both split_lo and split_hi, or neither"};
+        if (bc == PERIODIC && split_lo != 0) return {1, "periodic split must have split_lo == 0"};
+        cands.push_back({split_lo, split_hi});
+    } else if (bc == PERIODIC) {
+        int kl = 0, ku = 0;
+        for (int i = 0; i < n; ++i)
+            for (int c : P.A[i].col) {
+                long o = lmod(c - i, n);
+                if (o > n / 2) o -= n;
+                kl = std::max<long>(kl, -o);
+                ku = std::max<long>(ku, o);
+            }
+        for (int k = std::max(kl, ku); k <= std::min(n, KMAX_DELTA); ++k) cands.push_back({0, k});
+    } else {
+        // score candidates by (kernel band K, kl+ku, k)
+        const int lo0 = (bc == HERMITE) ? P.nbc : 0;
+        struct C { int K, bw, k, a, b; };
+        std::vector<C> cs;
+        for (int a = lo0; a <= lo0 + p + 1; ++a)
+            for (int b = lo0; b <= lo0 + p + 1; ++b) {
+                if (a + b > KMAX_DELTA || a + b >= n) continue;
+                int kl = 0, ku = 0;
+                for (int i = a; i < n - b; ++i)
+                    for (int c : P.A[i].col)
+                        if (c >= a && c < n - b) { kl = std::max(kl, i - c); ku = std::max(ku, c - i); }
+                cs.push_back({std::max(1, std::max(kl, ku)), kl + ku, a + b, a, b});
+            }
+        std::sort(cs.begin(), cs.end(), [](const C &x, const C &y) {
+            if (x.K != y.K) return x.K < y.K;
+            if (x.bw != y.bw) return x.bw < y.bw;
+            if (x.k != y.k) return x.k < y.k;
+            return std::abs(x.a - x.b) < std::abs(y.a - y.b);
+        });
+        for (auto &c : cs) cands.push_back({c.a, c.b});
+    }
+    if (n <= KMAX_DELTA) cands.push_back({0, n});  // tiny: dense delta' only
+    std::string why = "no admissible Schur split";
+    int why_code = 2;
+    std::mt19937_64 gen(12345);
+    std::uniform_real_distribution<double> U(-1.0, 1.0);
+    for (auto &c : cands) {
+        SplitResult r = try_split(P, c.first, c.second);
+        if (r.code) { why = r.msg; why_code = r.code; continue; }
+        build_segments(P, Lmax);
+        // self-check: residual of the equilibrated system with 4 random RHS
+        const int nb = 4;
+        std::vector<double> b((size_t)n * nb), x;
+        for (auto &v : b) v = U(gen);
+        x = b;
+        plan_solve_cpu(P, x.data(), nb, 1, nb);
+        double res = 0.0, bmax = 0.0;
+        for (int rr = 0; rr < nb; ++rr)
+            for (int i = 0; i < n; ++i) {
+                double acc = 0.0;
+                for (size_t e = 0; e < P.A[i].col.size(); ++e) acc += P.A[i].val[e] * x[(size_t)P.A[i].col[e] * nb + rr];
+                double bi = b[(size_t)i * nb + rr] * P.rowscale[i];
+                res = std::max(res, std::fabs(acc - bi));
+                bmax = std::max(bmax, std::fabs(bi));
+            }
+        if (res <= 1e-13 * bmax) return {0, ""};
+        why = "self-check residual too large for split";
+        why_code = 2;
+    }
+    return {why_code, why};
+}
+
+}  // namespace sb

@@ -1,0 +1,85 @@
+// plan.hpp -- host-side "create" step of the spline builder: collocation
+// matrix, Schur split, one-time factorisation, COO corners and the segment
+// coupling data of the in-CTA parallel recurrence.
+//
+// "the factorization is only done once at
+// initialization ... we take advantage of existing CPU libraries to
+// factorize the matrix and copy the result to the device".  There is no
+// LAPACK on the target box, so the banded factorisations (pttrf / pbtrf /
+// gbtrf-without-interchanges, getrf for delta') are written here.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace sb {
+
+enum Bc { PERIODIC = 0, GREVILLE = 1, HERMITE = 2 };
+enum QType { Q_PTTRS = 0, Q_PBTRS = 1, Q_GBTRS = 2 };
+
+constexpr int KMAX_BAND = 4;    // largest Q half-band the kernels are built for
+constexpr int KMAX_DELTA = 32;  // largest delta' order
+constexpr double BETA_DROP = 1e-14;  // keep |beta| > 1e-14 (DESIGN R4)
+
+struct SparseRow {
+    std::vector<int> col;
+    std::vector<double> val;
+};
+
+struct Plan {
+    // ---- spline space
+    int p = 0, bc = 0, N = 0, n = 0, nbc = 0;
+    std::vector<double> h;          // cell widths
+    std::vector<SparseRow> A;       // equilibrated collocation matrix rows
+    std::vector<double> rowscale;   // A_eq = diag(rowscale) * A_raw
+    // ---- Schur split (Eq. 3)
+    int s_lo = 0, s_hi = 0, k = 0, nQ = 0;
+    std::vector<int> drow;          // delta index -> row of A
+    int kl = 0, ku = 0, K = 1;      // Q band, kernel band (max, >=1)
+    int qtype = Q_GBTRS;
+    double growth = 0.0;
+    // ---- factors of Q in Q-local indices (forward unit-lower L, backward
+    // x_i = y_i*dinv_i - sum_m up_{i,m} x_{i+m})
+    std::vector<double> Lb;         // nQ*K : Lb[i*K+m-1] = L(i, i-m)
+    std::vector<double> Ub;         // nQ*K : Ub[i*K+m-1] = U(i, i+m)/U(i,i)
+    std::vector<double> dinv;       // nQ
+    // ---- corners
+    std::vector<double> beta_full;  // nQ*k, beta = Q^{-1} gamma (Eq. 4)
+    std::vector<int> lam_r, lam_c;  std::vector<double> lam_v;   // lambda COO
+    std::vector<int> beta_r, beta_c; std::vector<double> beta_v; // beta COO (thresholded)
+    std::vector<double> dprime;     // k*k delta' = delta - lambda beta
+    std::vector<double> dlu;        // k*k LU of delta' (getrf, partial pivoting)
+    std::vector<int> dpiv;          // k
+    // ---- in-CTA segments of the Q recurrences
+    int Lmax = 32, S = 1, seg_base = 0, seg_rem = 0, Lseg = 0;
+    std::vector<double> gspk;       // nQ*K forward spikes
+    std::vector<double> hspk;       // nQ*K backward spikes
+    int carry_f = 0, carry_b = 0;
+    // ---- head / tail windows holding every lambda column and beta row
+    int Wh = 0, Wt = 0;
+
+    int seg_start(int s) const { return s * seg_base + (s < seg_rem ? s : seg_rem); }
+    int seg_len(int s) const { return seg_base + (s < seg_rem ? 1 : 0); }
+    int win_slot(int qrow) const {  // -1 if outside the windows
+        if (qrow < Wh) return qrow;
+        if (qrow >= nQ - Wt) return Wh + (qrow - (nQ - Wt));
+        return -1;
+    }
+};
+
+// status codes mirror include/spline_builder.h
+struct Status {
+    int code = 0;
+    std::string msg;
+};
+
+// Build the spline space, the (equilibrated) collocation matrix, choose the
+// split, factor, compute corners and segment data.  split_lo/hi = -1: default.
+Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi,
+                  int Lmax);
+
+// Algorithm 1 on the CPU with the plan's factors (serial, fp64): reference
+// used by create's self-check and exported for tests.
+void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, int64_t pstride);
+
+}  // namespace sb

@@ -1,0 +1,183 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs (BASELINE.json tolerances):
+max relative coefficient error <= 1e-12 (fp64) / 1e-5 (fp32), interpolation
+residual <= 1e-12 (fp64).  Run on a B200 with ``pytest -m gpu``.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from oracle import GREVILLE, HERMITE, PERIODIC, Oracle, rel_coef_error
+from paper_conf_sc_asahilbpbgo24_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+
+TOL64 = 1e-12
+TOL32 = 1e-5
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def make(p, n_points, bc, kind):
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder
+    N = inputs.n_cells(p, n_points, bc)
+    x = inputs.breakpoints(N, kind)
+    return SplineBuilder(p, n_points, bc, x), Oracle(p, n_points, bc, x)
+
+
+def gpu_solve(torch, sb, b, dtype=None):
+    t = torch.from_numpy(b if dtype is None else b.astype(dtype)).cuda()
+    sb.solve_(t)
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+CASES = [
+    # (degree, n_points, bc, mesh)
+    (3, 16, PERIODIC, "uniform"),      # C1
+    (3, 1000, PERIODIC, "uniform"),    # C2 shape
+    (4, 1000, PERIODIC, "uniform"),
+    (5, 1000, PERIODIC, "uniform"),
+    (3, 1000, PERIODIC, "sin"),
+    (4, 1000, PERIODIC, "jitter"),
+    (5, 1000, PERIODIC, "jitter"),
+    (5, 1000, GREVILLE, "sin"),        # C3 Greville
+    (5, 996, HERMITE, "sin"),          # C3 Hermite
+    (3, 1024, PERIODIC, "uniform"),    # C4 shape
+    (3, 200, GREVILLE, "jitter"),
+    (3, 200, HERMITE, "uniform"),
+    (4, 200, HERMITE, "sin"),
+    (1, 50, PERIODIC, "uniform"),
+    (2, 50, PERIODIC, "jitter"),
+    (2, 40, GREVILLE, "sin"),
+    (3, 5, PERIODIC, "uniform"),
+    (5, 8, GREVILLE, "uniform"),
+    (3, 33, PERIODIC, "uniform"),
+    (3, 64, PERIODIC, "jitter"),
+]
+
+
+@pytest.mark.parametrize("case", CASES, ids=[f"p{c[0]}-n{c[1]}-bc{c[2]}-{c[3]}" for c in CASES])
+@pytest.mark.parametrize("batch", [1, 37, 256, 1000])
+def test_parity_fp64_batch_contiguous(torch_cuda, case, batch):
+    p, npts, bc, kind = case
+    sb, o = make(p, npts, bc, kind)
+    b = inputs.rhs(sb.n, batch, seed=1234 + batch, degree=p, bc=bc)
+    ref = o.solve(b)
+    got = gpu_solve(torch_cuda, sb, b)
+    err = rel_coef_error(got, ref)
+    assert err <= TOL64, (case, batch, err)
+    assert o.residual(got, b) <= TOL64
+
+
+@pytest.mark.parametrize("case", [c for c in CASES if c[1] >= 16][:10])
+def test_parity_fp32(torch_cuda, case):
+    p, npts, bc, kind = case
+    sb, o = make(p, npts, bc, kind)
+    b = inputs.rhs(sb.n, 300, seed=77, degree=p, bc=bc)
+    b32 = b.astype(np.float32)
+    ref = o.solve(b32.astype(np.float64))  # oracle on the fp32-rounded inputs
+    got = gpu_solve(torch_cuda, sb, b32)
+    assert got.dtype == np.float32
+    assert rel_coef_error(got.astype(np.float64), ref) <= TOL32
+
+
+@pytest.mark.parametrize("n_points,dtype", [(1024, np.float64), (1024, np.float32), (1000, np.float64)])
+def test_parity_point_contiguous(torch_cuda, n_points, dtype):
+    """C4 layout: x contiguous, batch_stride = n (transpose path)."""
+    torch = torch_cuda
+    sb, o = make(3, n_points, PERIODIC, "uniform")
+    f = inputs.gysela_slice(4, 8, 4, n_points, dtype=np.float64).reshape(-1, n_points)  # (batch, n)
+    ref = o.solve(np.ascontiguousarray(f.T.astype(dtype).astype(np.float64)))
+    t = torch.from_numpy(np.ascontiguousarray(f.astype(dtype))).cuda()
+    sb.solve_(t)  # (batch, n) -> point-contiguous
+    torch.cuda.synchronize()
+    got = t.cpu().numpy().T.astype(np.float64)
+    assert rel_coef_error(got, ref) <= (TOL64 if dtype == np.float64 else TOL32)
+
+
+def test_strided_equals_contiguous_bitwise(torch_cuda):
+    """The same RHS in batch-contiguous and point-contiguous layouts give the
+    same bits (same per-RHS arithmetic)."""
+    torch = torch_cuda
+    sb, _ = make(3, 1024, PERIODIC, "uniform")
+    b = inputs.rhs(sb.n, 96, seed=5)
+    t1 = torch.from_numpy(b).cuda()
+    t2 = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()
+    sb.solve_(t1)
+    sb.solve_(t2)
+    torch.cuda.synchronize()
+    assert torch.equal(t1, t2.t())
+
+
+def test_general_strided_subslice(torch_cuda):
+    """_strided: a sub-slice of a wider array (ld != batch), untouched columns
+    unchanged."""
+    torch = torch_cuda
+    sb, o = make(3, 1000, PERIODIC, "uniform")
+    b = inputs.rhs(sb.n, 500, seed=9)
+    t = torch.from_numpy(b).cuda()
+    view = t[:, 100:300]
+    sb.solve_strided_(view, batch=200, batch_stride=1, point_stride=500)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    assert np.array_equal(got[:, :100], b[:, :100]) and np.array_equal(got[:, 300:], b[:, 300:])
+    assert rel_coef_error(got[:, 100:300], o.solve(b[:, 100:300])) <= TOL64
+
+
+def test_batch_zero_and_errors(torch_cuda):
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, SplineBuilderError
+    sb = SplineBuilder(3, 100, PERIODIC)
+    t = torch.zeros(100, 0, dtype=torch.float64, device="cuda")
+    sb.solve_(t)
+    with pytest.raises(SplineBuilderError):
+        sb.solve_strided_(torch.zeros(100, 10, dtype=torch.float64, device="cuda"), 10, 3, 5)
+
+
+def test_solve_host_end_to_end(torch_cuda):
+    torch = torch_cuda
+    sb, o = make(3, 1000, PERIODIC, "uniform")
+    b = inputs.rhs(sb.n, 3001, seed=11)
+    pinned = torch.from_numpy(b.copy()).pin_memory()
+    sb.solve_host_(pinned)
+    assert rel_coef_error(pinned.numpy(), o.solve(b)) <= TOL64
+
+
+def test_c2_full_size_sampled(torch_cuda):
+    """C2 at full size (n=1000, 1e5 RHS) in the bench's launch configuration,
+    compared on a seeded sample of RHS (incl. first/last) + residual."""
+    torch = torch_cuda
+    sb, o = make(3, 1000, PERIODIC, "uniform")
+    B = 100000
+    b = inputs.rhs(sb.n, B, seed=1234)
+    t = torch.from_numpy(b).cuda()
+    sb.solve_(t)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    idx = np.unique(np.concatenate([[0, B - 1], np.random.default_rng(3).choice(B, 2048, replace=False)]))
+    ref = o.solve(np.ascontiguousarray(b[:, idx]))
+    assert rel_coef_error(got[:, idx], ref) <= TOL64
+    assert o.residual(got[:, idx], b[:, idx]) <= TOL64
+
+
+@pytest.mark.parametrize("bc,npts", [(GREVILLE, 1000), (HERMITE, 996)])
+def test_c3_full_size_sampled(torch_cuda, bc, npts):
+    torch = torch_cuda
+    sb, o = make(5, npts, bc, "sin")
+    B = 100000
+    b = inputs.rhs(sb.n, B, seed=4321, degree=5, bc=bc)
+    t = torch.from_numpy(b).cuda()
+    sb.solve_(t)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    idx = np.unique(np.concatenate([[0, B - 1], np.random.default_rng(4).choice(B, 1024, replace=False)]))
+    ref = o.solve(np.ascontiguousarray(b[:, idx]))
+    assert rel_coef_error(got[:, idx], ref) <= TOL64
+    assert o.residual(got[:, idx], b[:, idx]) <= TOL64
