@@ -1,0 +1,345 @@
+#!/usr/bin/env python
+"""Benchmark of the batched spline-coefficient build (BASELINE.json metric:
+"RHS/s and achieved HBM GB/s (% of peak), cubic n=1000, 1e5 RHS, fp64").
+
+A step = one in-place solve (Algorithm 1) of the whole
+batch of one workload: default C2 = cubic uniform periodic, n = 1000,
+1e5 RHS, fp64, batch-contiguous -- the configuration BASELINE.json's metric
+is quoted on.  Inputs (800 MB) are larger than L2 (126 MB); solves are timed
+in chunks of 40 back-to-back launches, the input restored and L2 flushed
+between chunks outside the CUDA events.
+
+  python bench.py [--gpus N --steps K --warmup W] [--workload C2|C3G|C3H|C4|C4F32|C5|C1]
+  python bench.py --impl reference ...   # the CPU oracle, same metric/config
+
+Multi-GPU (torchrun, one rank per GPU): weak scaling, each rank solves its
+own slice [rank*B, (rank+1)*B) of a global batch (RHS index drives the RNG);
+no collective on the data path, NCCL only for the barrier and the max-time
+reduction.  Prints one JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_sc_asahilbpbgo24_b200 import inputs  # noqa: E402
+
+METRIC = "RHS/s and achieved HBM GB/s (% of peak), cubic n=1000, 1e5 RHS, fp64"
+
+WORKLOADS = {
+    # name: (degree, n_points, bc, mesh, batch per GPU, dtype, layout, description)
+    "C1": (3, 16, 0, "uniform", 8, "f64", "batch", "C1 cubic uniform periodic n=16 batch=8 fp64"),
+    "C2": (3, 1000, 0, "uniform", 100000, "f64", "batch",
+           "C2 cubic uniform periodic n=1000 batch=1e5 fp64 batch-contiguous"),
+    "C3G": (5, 1000, 1, "sin", 100000, "f64", "batch", "C3 degree-5 non-uniform (sin map) Greville n=1000 batch=1e5 fp64"),
+    "C3H": (5, 996, 2, "sin", 100000, "f64", "batch", "C3 degree-5 non-uniform (sin map) Hermite n=1000 batch=1e5 fp64"),
+    "C4": (3, 1024, 0, "uniform", 131072, "f64", "point",
+           "C4 GYSELA slice f[64][64][32][x=1024] cubic periodic along x, x contiguous, fp64"),
+    "C4F32": (3, 1024, 0, "uniform", 131072, "f32", "point",
+              "C4 GYSELA slice f[64][64][32][x=1024] cubic periodic along x, x contiguous, fp32"),
+    "C5": (3, 1000, 0, "uniform", 1000000, "f64", "batch",
+           "C5 cubic uniform periodic n=1000, 1e6 RHS per GPU (8e6 over 8 GPUs) fp64"),
+}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def load_traffic(workload):
+    """dram bytes per launch from the committed ncu --set full capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p))
+    w = d.get(workload)
+    return None if w is None else w.get("dram_bytes_per_launch")
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons during the timed region
+    (streaming `nvidia-smi -lms`, the recipe's clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,power.draw")
+
+    def __init__(self, index=0, interval_ms=50):
+        self.index = index
+        self.interval_ms = interval_ms
+        self.samples = []
+        self._p = None
+        self._t = None
+
+    def _read(self):
+        for line in self._p.stdout:
+            parts = [x.strip() for x in line.strip().split(",")]
+            if len(parts) == 7:
+                self.samples.append(parts)
+
+    def __enter__(self):
+        try:
+            self._p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                        "--format=csv,noheader,nounits", f"-lms={self.interval_ms}"],
+                                       stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self._t = threading.Thread(target=self._read, daemon=True)
+            self._t.start()
+            time.sleep(0.3)  # first samples before the timed region starts
+        except Exception:
+            self._p = None
+        return self
+
+    def __exit__(self, *a):
+        if self._p is not None:
+            time.sleep(0.1)
+            self._p.terminate()
+            try:
+                self._p.wait(timeout=5)
+            except Exception:
+                self._p.kill()
+            self._t.join(timeout=5)
+
+    def summary(self):
+        def num(x):
+            try:
+                return float(x)
+            except ValueError:
+                return None
+        sm = [num(s[0]) for s in self.samples if num(s[0]) is not None]
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        mx = [num(s[1]) for s in self.samples if num(s[1]) is not None]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[2 + i].lower() == "active"})
+        pw = [num(s[6]) for s in self.samples if num(s[6]) is not None]
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(self.samples), "power_w_max": max(pw) if pw else None}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def make_rhs(deg, n, bc, B, first, layout, dtype):
+    b = inputs.rhs(n, B, seed=1234, degree=deg, bc=bc, first=first)  # (n, B) fp64
+    if layout == "point":
+        b = np.ascontiguousarray(b.T)
+    return np.ascontiguousarray(b.astype(np.float32 if dtype == "f32" else np.float64))
+
+
+def cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0, max_rhs=None):
+    """Time the oracle as it stands on a bounded sample; returns (RHS/s,
+    threads, sample description)."""
+    import oracle
+    o = oracle.Oracle(deg, npts, bc, knots)
+    threads = len(os.sched_getaffinity(0))
+    probe = 256
+    b = inputs.rhs(n, probe, seed=99, degree=deg, bc=bc)
+    t0 = time.perf_counter()
+    o.solve_(b.copy(), nthreads=threads)
+    dt = time.perf_counter() - t0
+    m = int(max(probe, min(target_s / max(dt, 1e-6) * probe, 200000)))
+    if max_rhs:
+        m = min(m, max_rhs)
+    b = inputs.rhs(n, m, seed=98, degree=deg, bc=bc)
+    t0 = time.perf_counter()
+    o.solve_(b, nthreads=threads)
+    dt = time.perf_counter() - t0
+    return m / dt, threads, f"{m} RHS of the same workload (n={n}), dense GEPP oracle, {threads} OpenMP threads"
+
+
+def run_reference(args, wl):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    deg, npts, bc, mesh, B, dt, layout, desc = wl
+    n = inputs.nbasis(deg, npts, bc)
+    knots = inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh)
+    import oracle
+    o = oracle.Oracle(deg, npts, bc, knots)
+    threads = len(os.sched_getaffinity(0))
+    # each step: a bounded sample sized so the whole run stays within minutes
+    rate0, _, _ = cpu_oracle_rate(deg, npts, bc, knots, n, target_s=2.0)
+    per_step = max(64, int(rate0 * min(4.0, 120.0 / max(1, args.steps + args.warmup))))  # whole run ~2 min
+    b0 = inputs.rhs(n, per_step, seed=1234, degree=deg, bc=bc)
+    for _ in range(args.warmup):
+        o.solve_(b0.copy(), nthreads=threads)
+    times = []
+    for _ in range(args.steps):
+        b = b0.copy()
+        t0 = time.perf_counter()
+        o.solve_(b, nthreads=threads)
+        times.append(time.perf_counter() - t0)
+    t = float(np.mean(times))
+    val = per_step / t
+    esz = 4 if dt == "f32" else 8
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "RHS/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": dt, "data": "synthetic",
+        "config": {"workload": desc, "n": n, "batch_per_step": per_step, "degree": deg, "bc": bc},
+        "achieved_gbs": val * 2 * n * esz / 1e9,
+        "cpu_baseline": {"value": val, "unit": "RHS/s", "cores": threads, "kind": "oracle",
+                         "sample": f"{per_step} RHS per step of the workload (n={n}); the full batch would take "
+                                   f"{B / val:.1f} s"},
+        "e2e": {"value": val, "unit": "RHS/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+    wl = WORKLOADS[args.workload]
+    if args.impl == "reference":
+        return run_reference(args, wl)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder
+
+    ws, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    deg, npts, bc, mesh, B, dt, layout, desc = wl
+    n = inputs.nbasis(deg, npts, bc)
+    knots = inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh)
+    sb = SplineBuilder(deg, npts, bc, knots)
+    esz = 4 if dt == "f32" else 8
+    # this rank's slice of the global batch (weak scaling)
+    host = make_rhs(deg, n, bc, B, rank * B, layout, dt)
+    pristine = torch.from_numpy(host).cuda()
+    x = pristine.clone()
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # The solve is in place, so repeated solves compute A^-k b, which grows
+    # like cond(A)^k: time chunks of CHUNK back-to-back solves, restoring the
+    # input and flushing L2 (256 MB write) between chunks, outside the events.
+    CHUNK = 40
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    for _ in range(args.warmup):
+        sb.solve_(x)
+    barrier()
+    nchunks = (args.steps + CHUNK - 1) // CHUNK
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(nchunks)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(nchunks)]
+    with ClockSampler(local) as clk:
+        barrier()
+        done = 0
+        for c in range(nchunks):
+            m = min(CHUNK, args.steps - done)
+            x.copy_(pristine)
+            flush.fill_(c & 0xFF)
+            starts[c].record(stream)
+            for _ in range(m):
+                sb.solve_(x)  # one fused kernel launch per step
+            ends[c].record(stream)
+            done += m
+        barrier()
+    total_ms = float(sum(s.elapsed_time(e) for s, e in zip(starts, ends)))
+    t_tensor = torch.tensor([total_ms, total_ms / args.steps], device="cuda", dtype=torch.float64)
+    if ws > 1:
+        dist.all_reduce(t_tensor, op=dist.ReduceOp.MAX)
+    total_ms, kern_avg_ms = float(t_tensor[0]), float(t_tensor[1])
+    ms_per_step = total_ms / args.steps
+    value = ws * B / (ms_per_step / 1e3)
+    alg_bytes = 2.0 * n * B * esz
+    achieved = alg_bytes / (kern_avg_ms / 1e3) / 1e9
+    peak, peak_kind = load_peaks()
+
+    # end to end through the C ABI with host buffers (pinned), copies in the timed region
+    e2e = None
+    if not args.no_e2e:
+        hp = torch.from_numpy(host.copy()).pin_memory()
+        if layout == "batch":
+            sb.solve_host_(hp)  # warm-up (allocates staging)
+            barrier()
+            ts = []
+            for _ in range(args.e2e_steps):
+                hp.copy_(torch.from_numpy(host))
+                barrier()
+                t0 = time.perf_counter()
+                sb.solve_host_(hp)
+                ts.append(time.perf_counter() - t0)
+            te = torch.tensor([float(np.mean(ts))], device="cuda", dtype=torch.float64)
+            if ws > 1:
+                dist.all_reduce(te, op=dist.ReduceOp.MAX)
+            e2e = {"value": ws * B / float(te[0]), "unit": "RHS/s", "h2d_bytes_per_step": int(host.nbytes),
+                   "d2h_bytes_per_step": int(host.nbytes), "path": "spline_builder_solve_host (pinned, chunked)"}
+        else:
+            # point-contiguous: H2D copy + solve + D2H copy on the current stream
+            dev = torch.empty_like(pristine)
+            ts = []
+            for _ in range(args.e2e_steps + 1):
+                barrier()
+                t0 = time.perf_counter()
+                dev.copy_(hp, non_blocking=True)
+                sb.solve_(dev)
+                hp.copy_(dev, non_blocking=True)
+                torch.cuda.synchronize()
+                ts.append(time.perf_counter() - t0)
+            e2e = {"value": ws * B / float(np.mean(ts[1:])), "unit": "RHS/s", "h2d_bytes_per_step": int(host.nbytes),
+                   "d2h_bytes_per_step": int(host.nbytes), "path": "H2D + spline_builder_solve + D2H"}
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        rate, cores, sample = cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0)
+        cpu = {"value": rate, "unit": "RHS/s", "cores": cores, "kind": "oracle", "sample": sample}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "RHS/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": dt, "data": "synthetic (Philox U(-1,1) RHS, seeded)",
+            "config": {"workload": desc, "n": n, "batch_per_gpu": B, "degree": deg, "bc": ["periodic", "greville",
+                                                                                        "hermite"][bc],
+                       "mesh": mesh, "layout": "batch-contiguous" if layout == "batch" else "point-contiguous",
+                       "l2": f"inputs {host.nbytes / 1e6:.0f} MB per GPU > 126 MB L2; input restored + 256 MB L2 flush every 40 steps (untimed)",
+                       "parallelism": f"dp{ws} (RHS shards)"},
+            "achieved_gbs": achieved, "pct_of_8tbs": achieved / 8000.0,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": load_traffic(args.workload),
+                         "peak_kind": peak_kind, "kernel_ms": kern_avg_ms,
+                         "algorithmic_bytes_per_launch": alg_bytes},
+            "clocks": clk.summary(),
+            "e2e": e2e,
+            "gpu_launches": args.steps,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

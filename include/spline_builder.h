@@ -134,7 +134,10 @@ typedef struct {
                                        2 gbtrs (general band, no interchanges)   */
     int nnz_lambda, nnz_beta;       /* COO sizes; beta kept if > 1e-14   */
     int beta_rows_head, beta_rows_tail; /* Q rows at each end touched by beta     */
-    int n_segments, seg_len;        /* in-CTA segment split of the Q recurrences  */
+    int nnz_Lambda, nnz_gamma;      /* Lambda = lambda Q^-1 (kept if > 1e-14) and
+                                       gamma: the corner data the kernel uses      */
+    int n_segments, seg_len;        /* in-CTA segment split of the Q recurrences
+                                       (fp64 kernels)                             */
     int carry_fwd, carry_bwd;       /* predecessor segments in the carry walks    */
     double max_pivot_growth;        /* max |U| / max |Q| of the no-pivot LU        */
 } spline_builder_info_t;

@@ -29,7 +29,8 @@ EXPORTS = [
 class SplineBuilderInfo(ctypes.Structure):
     _fields_ = [(name, ctypes.c_int) for name in (
         "degree", "bc", "n_cells", "nbasis", "split_lo", "split_hi", "k", "q_kl", "q_ku", "q_type",
-        "nnz_lambda", "nnz_beta", "beta_rows_head", "beta_rows_tail", "n_segments", "seg_len",
+        "nnz_lambda", "nnz_beta", "beta_rows_head", "beta_rows_tail", "nnz_Lambda", "nnz_gamma", "n_segments",
+        "seg_len",
         "carry_fwd", "carry_bwd")] + [("max_pivot_growth", ctypes.c_double)]
 
     def as_dict(self):

@@ -27,7 +27,6 @@ int fail(int code, const std::string &msg) {
     return code;
 }
 
-constexpr int LMAX_SEG = 32;  // must match the kernels' register segment length
 
 }  // namespace
 
@@ -67,48 +66,41 @@ std::vector<C> conv(const std::vector<double> &v) {
 
 int upload(spline_builder *h) {
     const sb::Plan &P = h->plan;
-    const int K = P.K, nQ = P.nQ, k = P.k, W = P.Wh + P.Wt;
-    const int FS = 2 * K, BS = 2 * K + 2;
-    std::vector<double> fwd((size_t)nQ * FS, 0.0), bwd((size_t)nQ * BS, 0.0);
+    const int K = P.K, nQ = P.nQ, k = P.k;
+    // padded SoA factor arrays: stride nQpa covers both segment plans
+    const int nQpa = std::max(std::max(P.seg[0].nQp, P.seg[1].nQp), 2);
+    std::vector<double> Lr((size_t)K * nQpa, 0.0), Ur((size_t)K * nQpa, 0.0), dinv(nQpa, 1.0);
     for (int i = 0; i < nQ; ++i) {
         for (int m = 0; m < K; ++m) {
-            fwd[(size_t)i * FS + m] = P.Lb[(size_t)i * K + m];
-            fwd[(size_t)i * FS + K + m] = P.gspk[(size_t)i * K + m];
-            bwd[(size_t)i * BS + 1 + m] = P.Ub[(size_t)i * K + m];
-            bwd[(size_t)i * BS + 1 + K + m] = P.hspk[(size_t)i * K + m];
+            Lr[(size_t)m * nQpa + i] = P.Lb[(size_t)i * K + m];
+            Ur[(size_t)m * nQpa + i] = P.Ub[(size_t)i * K + m];
         }
-        bwd[(size_t)i * BS] = P.dinv[i];
-    }
-    // dense thresholded beta rows over the head/tail windows (COO semantic)
-    std::vector<double> betaW((size_t)W * k, 0.0);
-    for (size_t e = 0; e < P.beta_v.size(); ++e) {
-        int slot = P.win_slot(P.beta_r[e]);
-        if (slot < 0) return fail(SB_UNSUPPORTED, "internal: beta row outside window");
-        betaW[(size_t)slot * k + P.beta_c[e]] = P.beta_v[e];
-    }
-    std::vector<int> lam_slot(P.lam_c.size());
-    for (size_t e = 0; e < P.lam_c.size(); ++e) {
-        lam_slot[e] = P.win_slot(P.lam_c[e]);
-        if (lam_slot[e] < 0) return fail(SB_UNSUPPORTED, "internal: lambda column outside window");
+        dinv[i] = P.dinv[i];
     }
     std::vector<double> dscale(k);
     for (int d = 0; d < k; ++d) dscale[d] = P.rowscale[P.drow[d]];
-
+    // gamma entries of each segment (COO sorted by Q row)
+    std::vector<int> gptr[2];
+    for (int c = 0; c < 2; ++c) {
+        const sb::SegPlan &G = P.seg[c];
+        gptr[c].assign(G.S + 1, 0);
+        for (int s = 0, e = 0; s <= G.S; ++s) {
+            while (e < (int)P.gam_r.size() && P.gam_r[e] < s * G.L) ++e;
+            gptr[c][s] = e;
+        }
+        gptr[c][G.S] = (int)P.gam_r.size();
+    }
     Packer pk;
-    size_t o_fwd[2], o_bwd[2], o_beta[2], o_lamv[2], o_dlu[2], o_ds[2];
-    o_fwd[0] = pk.addv(fwd);
-    o_bwd[0] = pk.addv(bwd);
-    o_beta[0] = pk.addv(betaW);
-    o_lamv[0] = pk.addv(P.lam_v);
-    o_dlu[0] = pk.addv(P.dlu);
-    o_ds[0] = pk.addv(dscale);
-    o_fwd[1] = pk.addv(conv<float>(fwd));
-    o_bwd[1] = pk.addv(conv<float>(bwd));
-    o_beta[1] = pk.addv(conv<float>(betaW));
-    o_lamv[1] = pk.addv(conv<float>(P.lam_v));
-    o_dlu[1] = pk.addv(conv<float>(P.dlu));
-    o_ds[1] = pk.addv(conv<float>(dscale));
-    size_t o_lamr = pk.addv(P.lam_r), o_lams = pk.addv(lam_slot), o_dpiv = pk.addv(P.dpiv), o_drow = pk.addv(P.drow);
+    size_t oL[2], oU[2], oD[2], oLam[2], oGam[2], oDlu[2], oDs[2], oG[2], oH[2];
+    for (int c = 0; c < 2; ++c) {
+        auto put = [&](const std::vector<double> &v) { return c == 0 ? pk.addv(v) : pk.addv(conv<float>(v)); };
+        oL[c] = put(Lr); oU[c] = put(Ur); oD[c] = put(dinv);
+        oLam[c] = put(P.Lam_v); oGam[c] = put(P.gam_v); oDlu[c] = put(P.dlu); oDs[c] = put(dscale);
+        oG[c] = put(P.seg[c].G); oH[c] = put(P.seg[c].H);
+    }
+    size_t o_lamptr = pk.addv(P.Lam_ptr), o_lamc = pk.addv(P.Lam_c), o_gamr = pk.addv(P.gam_r),
+           o_gamc = pk.addv(P.gam_c), o_dpiv = pk.addv(P.dpiv), o_drow = pk.addv(P.drow);
+    size_t o_gptr[2] = {pk.addv(gptr[0]), pk.addv(gptr[1])};
     h->blob_bytes = std::max<size_t>(pk.bytes.size(), 16);
     cudaError_t e = cudaMalloc(&h->blob, h->blob_bytes);
     if (e != cudaSuccess) return fail(SB_NOMEM, std::string("cudaMalloc(blob): ") + cudaGetErrorString(e));
@@ -116,16 +108,18 @@ int upload(spline_builder *h) {
     if (e != cudaSuccess) return fail(SB_CUDA, std::string("cudaMemcpy(blob): ") + cudaGetErrorString(e));
     auto at = [&](size_t off) { return (const void *)((const unsigned char *)h->blob + off); };
     sb::DevPlan &d = h->dp;
-    d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K;
-    d.S = P.S; d.seg_base = P.seg_base; d.seg_rem = P.seg_rem;
-    d.carry_f = P.carry_f; d.carry_b = P.carry_b;
-    d.Wh = P.Wh; d.Wt = P.Wt; d.nlam = (int)P.lam_v.size();
-    d.fstride = FS; d.bstride = BS;
+    d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K; d.nQpa = nQpa;
+    d.lam_nnz = (int)P.Lam_v.size(); d.gam_nnz = (int)P.gam_v.size();
     for (int c = 0; c < 2; ++c) {
-        d.fwd[c] = at(o_fwd[c]); d.bwd[c] = at(o_bwd[c]); d.betaW[c] = at(o_beta[c]);
-        d.lam_v[c] = at(o_lamv[c]); d.dlu[c] = at(o_dlu[c]); d.dscale[c] = at(o_ds[c]);
+        d.Lr[c] = at(oL[c]); d.Ur[c] = at(oU[c]); d.dinv[c] = at(oD[c]);
+        d.lam_v[c] = at(oLam[c]); d.gam_v[c] = at(oGam[c]); d.dlu[c] = at(oDlu[c]); d.dscale[c] = at(oDs[c]);
+        const sb::SegPlan &G = P.seg[c];
+        d.seg[c].L = G.L; d.seg[c].S = G.S; d.seg[c].nQp = G.nQp;
+        d.seg[c].carry_f = G.carry_f; d.seg[c].carry_b = G.carry_b;
+        d.seg[c].G = at(oG[c]); d.seg[c].H = at(oH[c]); d.seg[c].gptr = (const int *)at(o_gptr[c]);
     }
-    d.lam_r = (const int *)at(o_lamr); d.lam_slot = (const int *)at(o_lams);
+    d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
+    d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);
     d.dpiv = (const int *)at(o_dpiv); d.drow = (const int *)at(o_drow);
     return 0;
 }
@@ -164,7 +158,7 @@ spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, cons
     spline_builder *h = new (std::nothrow) spline_builder();
     if (!h) { fail(SB_NOMEM, "out of host memory"); return nullptr; }
     try {
-        sb::Status st = sb::build_plan(h->plan, degree, n_points, bc, knots, split_lo, split_hi, LMAX_SEG);
+        sb::Status st = sb::build_plan(h->plan, degree, n_points, bc, knots, split_lo, split_hi);
         if (st.code) { fail(st.code, st.msg); delete h; return nullptr; }
     } catch (const std::bad_alloc &) {
         fail(SB_NOMEM, "out of host memory in create"); delete h; return nullptr;
@@ -282,10 +276,11 @@ int spline_builder_get_info(spline_builder_t h, spline_builder_info_t *info) {
     info->q_kl = P.kl; info->q_ku = P.ku; info->q_type = P.qtype;
     info->nnz_lambda = (int)P.lam_v.size(); info->nnz_beta = (int)P.beta_v.size();
     int head = 0, tail = 0;
-    for (int r : P.beta_r) { if (r < P.Wh) head = std::max(head, r + 1); else tail = std::max(tail, P.nQ - r); }
+    for (int r : P.beta_r) { if (r < P.nQ / 2) head = std::max(head, r + 1); else tail = std::max(tail, P.nQ - r); }
     info->beta_rows_head = head; info->beta_rows_tail = tail;
-    info->n_segments = P.S; info->seg_len = P.Lseg;
-    info->carry_fwd = P.carry_f; info->carry_bwd = P.carry_b;
+    info->nnz_Lambda = (int)P.Lam_v.size(); info->nnz_gamma = (int)P.gam_v.size();
+    info->n_segments = P.seg[0].S; info->seg_len = P.seg[0].L;
+    info->carry_fwd = P.seg[0].carry_f; info->carry_bwd = P.seg[0].carry_b;
     info->max_pivot_growth = P.growth;
     return SB_OK;
 }

@@ -6,23 +6,26 @@
 
 namespace sb {
 
-// Packed constant blob uploaded once at create ("copy the
-// result to the device").  Offsets are in bytes from the blob base; each
-// section is 16-byte aligned.  Both an fp64 and an fp32 copy of the
-// floating-point sections are stored (fp32 compute path).
-struct DevPlan {
-    int n, nQ, s_lo, k, K;          // order, Q order, Q offset, delta order, band
-    int S, seg_base, seg_rem;       // segments of the Q recurrences
-    int carry_f, carry_b;           // carry-walk depths
-    int Wh, Wt, nlam;               // window sizes, nnz(lambda)
-    // record strides (elements): forward = 2K (L, g), backward = 2K+2 (dinv, U', h, pad)
-    int fstride, bstride;
-    // device pointers (fp64 then fp32 copies)
-    const void *fwd[2], *bwd[2], *betaW[2], *lam_v[2], *dlu[2], *dscale[2];
-    const int *lam_r, *lam_slot, *dpiv, *drow;
+// segment plan of one compute precision (register segment length L)
+struct DevSeg {
+    int L, S, nQp, carry_f, carry_b;
+    const void *G, *H;    // S*K*K forward / backward transfer matrices (compute type)
+    const int *gptr;      // S+1: gamma COO entries of segment s are [gptr[s], gptr[s+1])
 };
 
-enum LayoutKind { LAYOUT_BATCH_CONTIG = 0, LAYOUT_STRIDED = 1 };
+// Packed constants uploaded once at create ("copy the result
+// to the device").  Floating-point sections exist in fp64 ([0]) and fp32 ([1]).
+struct DevPlan {
+    int n, nQ, s_lo, k, K;         // order, Q order, Q offset, delta order, kernel band
+    int nQpa;                      // stride of the padded factor arrays
+    int lam_nnz, gam_nnz;          // Lambda CSR / gamma COO sizes
+    const void *Lr[2];             // K arrays of nQpa: L(i, i-1-m) at [m*nQpa + i]
+    const void *Ur[2];             // K arrays of nQpa: U'(i, i+1+m) at [m*nQpa + i]
+    const void *dinv[2];           // nQpa (1 on padding rows)
+    const void *lam_v[2], *gam_v[2], *dlu[2], *dscale[2];
+    const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
+    DevSeg seg[2];                 // [0] fp64 kernels, [1] fp32 kernels
+};
 
 struct SolveArgs {
     void *rhs;
@@ -35,8 +38,5 @@ struct SolveArgs {
 
 // returns 0 on success, else an SB_* status; fills err on failure
 int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, int errlen);
-
-// bytes of dynamic shared memory the constant sections need (for validation)
-size_t const_smem_bytes(const DevPlan &P, int dtype);
 
 }  // namespace sb

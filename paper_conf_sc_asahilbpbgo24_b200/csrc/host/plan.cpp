@@ -242,10 +242,8 @@ SplitResult try_split(Plan &P, int slo, int shi) {
             qtype = Q_GBTRS;
         }
     }
-    // beta = Q^{-1} gamma (Eq. 4), one banded solve per delta column
-    std::vector<double> beta((size_t)nQ * k, 0.0), v(nQ);
-    for (int c = 0; c < k; ++c) {
-        for (int i = 0; i < nQ; ++i) v[i] = gam[(size_t)i * k + c];
+    // banded solves with the factors: Q v = w (in place) and Q^T v = w
+    auto qsolve = [&](std::vector<double> &v) {
         for (int i = 0; i < nQ; ++i)
             for (int m = 1; m <= K && i - m >= 0; ++m) v[i] -= Lb[(size_t)i * K + m - 1] * v[i - m];
         for (int i = nQ - 1; i >= 0; --i) {
@@ -253,7 +251,28 @@ SplitResult try_split(Plan &P, int slo, int shi) {
             for (int m = 1; m <= K && i + m < nQ; ++m) acc -= Ub[(size_t)i * K + m - 1] * v[i + m];
             v[i] = acc;
         }
+    };
+    // Q = L D (I + U'),  Q^T = (I + U')^T D L^T
+    auto qtsolve = [&](std::vector<double> &v) {
+        for (int j = 0; j < nQ; ++j)
+            for (int m = 1; m <= K && j - m >= 0; ++m) v[j] -= Ub[(size_t)(j - m) * K + m - 1] * v[j - m];
+        for (int j = 0; j < nQ; ++j) v[j] *= dinv[j];
+        for (int j = nQ - 1; j >= 0; --j)
+            for (int m = 1; m <= K && j + m < nQ; ++m) v[j] -= Lb[(size_t)(j + m) * K + m - 1] * v[j + m];
+    };
+    // beta = Q^{-1} gamma (Eq. 4), one banded solve per delta column
+    std::vector<double> beta((size_t)nQ * k, 0.0), v(nQ);
+    for (int c = 0; c < k; ++c) {
+        for (int i = 0; i < nQ; ++i) v[i] = gam[(size_t)i * k + c];
+        qsolve(v);
         for (int i = 0; i < nQ; ++i) beta[(size_t)i * k + c] = v[i];
+    }
+    // Lambda = lambda Q^{-1} (transposed twin of beta): Lambda_d^T = Q^{-T} lambda_d^T
+    std::vector<double> Lam((size_t)k * nQ, 0.0);
+    for (int d = 0; d < k; ++d) {
+        for (int i = 0; i < nQ; ++i) v[i] = lam[(size_t)d * nQ + i];
+        qtsolve(v);
+        for (int i = 0; i < nQ; ++i) Lam[(size_t)d * nQ + i] = v[i];
     }
     // delta' = delta - lambda beta (Eq. 4)
     std::vector<double> dp = del;
@@ -288,7 +307,6 @@ SplitResult try_split(Plan &P, int slo, int shi) {
     for (int d = 0; d < k; ++d) P.drow[d] = d < slo ? d : n - shi + (d - slo);
     P.kl = kl; P.ku = ku; P.K = K; P.qtype = qtype; P.growth = growth;
     P.Lb.swap(Lb); P.Ub.swap(Ub); P.dinv.swap(dinv);
-    P.beta_full.swap(beta);
     P.dprime = dp; P.dlu.swap(lu); P.dpiv.swap(piv);
     P.lam_r.clear(); P.lam_c.clear(); P.lam_v.clear();
     for (int r = 0; r < k; ++r)
@@ -296,81 +314,80 @@ SplitResult try_split(Plan &P, int slo, int shi) {
             if (lam[(size_t)r * nQ + i] != 0.0) {
                 P.lam_r.push_back(r); P.lam_c.push_back(i); P.lam_v.push_back(lam[(size_t)r * nQ + i]);
             }
+    P.gam_r.clear(); P.gam_c.clear(); P.gam_v.clear();
+    for (int i = 0; i < nQ; ++i)
+        for (int c = 0; c < k; ++c)
+            if (gam[(size_t)i * k + c] != 0.0) {
+                P.gam_r.push_back(i); P.gam_c.push_back(c); P.gam_v.push_back(gam[(size_t)i * k + c]);
+            }
     P.beta_r.clear(); P.beta_c.clear(); P.beta_v.clear();
     for (int i = 0; i < nQ; ++i)
         for (int c = 0; c < k; ++c) {
-            double b = P.beta_full[(size_t)i * k + c];
-            if (std::fabs(b) > BETA_DROP) { P.beta_r.push_back(i); P.beta_c.push_back(c); P.beta_v.push_back(b); }
+            double b = beta[(size_t)i * k + c];
+            if (std::fabs(b) > CORNER_DROP) { P.beta_r.push_back(i); P.beta_c.push_back(c); P.beta_v.push_back(b); }
         }
+    P.Lam_ptr.assign(k + 1, 0); P.Lam_c.clear(); P.Lam_v.clear();
+    for (int d = 0; d < k; ++d) {
+        for (int i = 0; i < nQ; ++i) {
+            double l = Lam[(size_t)d * nQ + i];
+            if (std::fabs(l) > CORNER_DROP) { P.Lam_c.push_back(i); P.Lam_v.push_back(l); }
+        }
+        P.Lam_ptr[d + 1] = (int)P.Lam_c.size();
+    }
     return R;
 }
 
-// segment partition + spike vectors + carry depths + windows
-void build_segments(Plan &P, int Lmax) {
+// segment partition of the padded Q for register segment length L: transfer
+// matrices of each segment and the carry-walk depths.
+void build_segplan(const Plan &P, SegPlan &G, int L) {
     const int nQ = P.nQ, K = P.K;
-    P.Lmax = Lmax;
-    int S = nQ > 0 ? (nQ + Lmax - 1) / Lmax : 1;
-    if (S > 1 && nQ / S < K) S = 1;
-    P.S = S;
-    P.seg_base = nQ / S;
-    P.seg_rem = nQ % S;
-    P.Lseg = P.seg_base + (P.seg_rem ? 1 : 0);
-    P.gspk.assign((size_t)nQ * K, 0.0);
-    P.hspk.assign((size_t)nQ * K, 0.0);
-    std::vector<double> y(nQ + 2 * K);
-    for (int s = 1; s < S; ++s) {
-        int a = P.seg_start(s), len = P.seg_len(s);
+    G.L = L;
+    G.S = nQ > 0 ? (nQ + L - 1) / L : 1;
+    G.nQp = G.S * L;
+    const int S = G.S;
+    auto Lf = [&](int row, int m) { return row < nQ ? P.Lb[(size_t)row * K + m - 1] : 0.0; };  // pad: identity
+    auto Uf = [&](int row, int m) { return row < nQ ? P.Ub[(size_t)row * K + m - 1] : 0.0; };
+    G.G.assign((size_t)S * K * K, 0.0);
+    G.H.assign((size_t)S * K * K, 0.0);
+    std::vector<double> y(L + 2 * K);
+    for (int t = 1; t < S; ++t) {  // forward: segment t's response to inflow unit m, at rows a+L-1-j
+        const int a = t * L;
         for (int m = 1; m <= K; ++m) {
-            // y indices shifted by K: y[K + i] = y_{a+i}, y[K - m'] = inflow state
-            std::fill(y.begin(), y.begin() + K + len, 0.0);
-            y[K - m] = 1.0;
-            for (int i = 0; i < len; ++i) {
-                int row = a + i;
+            std::fill(y.begin(), y.end(), 0.0);
+            y[K - m] = 1.0;  // y[K+i] = y_{a+i}
+            for (int i = 0; i < L; ++i) {
                 double acc = 0.0;
-                for (int mm = 1; mm <= K; ++mm) acc -= P.Lb[(size_t)row * K + mm - 1] * y[K + i - mm];
+                for (int mm = 1; mm <= K; ++mm) acc -= Lf(a + i, mm) * y[K + i - mm];
                 y[K + i] = acc;
-                P.gspk[(size_t)row * K + m - 1] = acc;
             }
+            for (int j = 0; j < K; ++j) G.G[((size_t)t * K + j) * K + (m - 1)] = y[K + L - 1 - j];
         }
     }
-    for (int s = 0; s + 1 < S; ++s) {
-        int a = P.seg_start(s), len = P.seg_len(s);
+    for (int t = 0; t + 1 < S; ++t) {  // backward: response to outflow unit m, at rows a+j
+        const int a = t * L;
         for (int m = 1; m <= K; ++m) {
-            // x[i] = x_{a+i}, i in [0, len+K)
-            std::fill(y.begin(), y.begin() + len + K, 0.0);
-            y[len + m - 1] = 1.0;
-            for (int i = len - 1; i >= 0; --i) {
-                int row = a + i;
+            std::fill(y.begin(), y.end(), 0.0);
+            y[L + m - 1] = 1.0;  // y[i] = x_{a+i}
+            for (int i = L - 1; i >= 0; --i) {
                 double acc = 0.0;
-                for (int mm = 1; mm <= K; ++mm) acc -= P.Ub[(size_t)row * K + mm - 1] * y[i + mm];
+                for (int mm = 1; mm <= K; ++mm) acc -= Uf(a + i, mm) * y[i + mm];
                 y[i] = acc;
-                P.hspk[(size_t)row * K + m - 1] = acc;
             }
+            for (int j = 0; j < K; ++j) G.H[((size_t)t * K + j) * K + (m - 1)] = y[j];
         }
     }
-    // carry depths: smallest T with prod ||G|| <= 2^-60 or reaching an exact end
+    // carry depths: smallest T with prod ||transfer||_inf <= 2^-60, or an exact end
     const double eps = std::ldexp(1.0, -60);
-    auto Gnorm = [&](int t) {  // forward transfer of segment t (rows at its end)
-        int end = P.seg_start(t) + P.seg_len(t);
-        double nrm = 0.0;
+    auto nrm = [&](const std::vector<double> &M, int t) {
+        double r = 0.0;
         for (int j = 0; j < K; ++j) {
             double s = 0.0;
-            for (int m = 0; m < K; ++m) s += std::fabs(P.gspk[(size_t)(end - 1 - j) * K + m]);
-            nrm = std::max(nrm, s);
+            for (int m = 0; m < K; ++m) s += std::fabs(M[((size_t)t * K + j) * K + m]);
+            r = std::max(r, s);
         }
-        return nrm;
+        return r;
     };
-    auto Hnorm = [&](int t) {
-        int a = P.seg_start(t);
-        double nrm = 0.0;
-        for (int j = 0; j < K; ++j) {
-            double s = 0.0;
-            for (int m = 0; m < K; ++m) s += std::fabs(P.hspk[(size_t)(a + j) * K + m]);
-            nrm = std::max(nrm, s);
-        }
-        return nrm;
-    };
-    P.carry_f = 0;
+    G.carry_f = 0;
     for (int s = 1; s < S; ++s) {
         int T = 0;
         double prod = 1.0;
@@ -378,12 +395,12 @@ void build_segments(Plan &P, int Lmax) {
             ++T;
             int t = s - T;
             if (t == 0) break;
-            prod *= Gnorm(t);
+            prod *= nrm(G.G, t);
             if (prod <= eps) break;
         }
-        P.carry_f = std::max(P.carry_f, T);
+        G.carry_f = std::max(G.carry_f, T);
     }
-    P.carry_b = 0;
+    G.carry_b = 0;
     for (int s = 0; s + 1 < S; ++s) {
         int T = 0;
         double prod = 1.0;
@@ -391,43 +408,27 @@ void build_segments(Plan &P, int Lmax) {
             ++T;
             int t = s + T;
             if (t == S - 1) break;
-            prod *= Hnorm(t);
+            prod *= nrm(G.H, t);
             if (prod <= eps) break;
         }
-        P.carry_b = std::max(P.carry_b, T);
+        G.carry_b = std::max(G.carry_b, T);
     }
-    // windows: every lambda column and beta row
-    int head = -1, tail = nQ;
-    auto note = [&](int q) {
-        if (q < nQ / 2 + 1) head = std::max(head, q);
-        else tail = std::min(tail, q);
-    };
-    for (int c : P.lam_c) note(c);
-    for (int r : P.beta_r) note(r);
-    P.Wh = head + 1;
-    P.Wt = nQ - tail;
-    if (P.Wh + P.Wt >= nQ) { P.Wh = nQ; P.Wt = 0; }
 }
 
 }  // namespace
 
 void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, int64_t pstride) {
-    const int n = P.n, nQ = P.nQ, k = P.k, K = P.K;
+    const int nQ = P.nQ, k = P.k, K = P.K;
     std::vector<double> v(nQ), x1(k);
     for (int64_t r = 0; r < batch; ++r) {
         double *col = rhs + r * bstride;
         for (int i = 0; i < nQ; ++i) v[i] = col[(int64_t)(P.s_lo + i) * pstride];
-        for (int d = 0; d < k; ++d) x1[d] = col[(int64_t)P.drow[d] * pstride] * P.rowscale[P.drow[d]];
-        // step 2: Q x0' = b0
-        for (int i = 0; i < nQ; ++i)
-            for (int m = 1; m <= K && i - m >= 0; ++m) v[i] -= P.Lb[(size_t)i * K + m - 1] * v[i - m];
-        for (int i = nQ - 1; i >= 0; --i) {
-            double acc = v[i] * P.dinv[i];
-            for (int m = 1; m <= K && i + m < nQ; ++m) acc -= P.Ub[(size_t)i * K + m - 1] * v[i + m];
-            v[i] = acc;
+        // x1 = delta'^{-1} (b1 - Lambda b0),  Lambda = lambda Q^{-1}
+        for (int d = 0; d < k; ++d) {
+            double acc = col[(int64_t)P.drow[d] * pstride] * P.rowscale[P.drow[d]];
+            for (int e = P.Lam_ptr[d]; e < P.Lam_ptr[d + 1]; ++e) acc -= P.Lam_v[e] * v[P.Lam_c[e]];
+            x1[d] = acc;
         }
-        // step 3: delta' x1 = b1 - lambda x0'
-        for (size_t e = 0; e < P.lam_v.size(); ++e) x1[P.lam_r[e]] -= P.lam_v[e] * v[P.lam_c[e]];
         for (int d = 0; d < k; ++d)
             if (P.dpiv[d] != d) std::swap(x1[d], x1[P.dpiv[d]]);
         for (int i = 1; i < k; ++i)
@@ -436,15 +437,21 @@ void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, 
             for (int j = i + 1; j < k; ++j) x1[i] -= P.dlu[(size_t)i * k + j] * x1[j];
             x1[i] /= P.dlu[(size_t)i * k + i];
         }
-        // step 4: x0 = x0' - beta x1
-        for (size_t e = 0; e < P.beta_v.size(); ++e) v[P.beta_r[e]] -= P.beta_v[e] * x1[P.beta_c[e]];
+        // x0 = Q^{-1} (b0 - gamma x1)
+        for (size_t e = 0; e < P.gam_v.size(); ++e) v[P.gam_r[e]] -= P.gam_v[e] * x1[P.gam_c[e]];
+        for (int i = 0; i < nQ; ++i)
+            for (int m = 1; m <= K && i - m >= 0; ++m) v[i] -= P.Lb[(size_t)i * K + m - 1] * v[i - m];
+        for (int i = nQ - 1; i >= 0; --i) {
+            double acc = v[i] * P.dinv[i];
+            for (int m = 1; m <= K && i + m < nQ; ++m) acc -= P.Ub[(size_t)i * K + m - 1] * v[i + m];
+            v[i] = acc;
+        }
         for (int i = 0; i < nQ; ++i) col[(int64_t)(P.s_lo + i) * pstride] = v[i];
         for (int d = 0; d < k; ++d) col[(int64_t)P.drow[d] * pstride] = x1[d];
     }
 }
 
-Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi,
-                  int Lmax) {
+Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi) {
     P = Plan();
     if (degree < 1 || degree > 5) return {1, "degree must be in 1..5"};
     if (bc != PERIODIC && bc != GREVILLE && bc != HERMITE) return {1, "unknown boundary condition"};
@@ -546,7 +553,8 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
     for (auto &c : cands) {
         SplitResult r = try_split(P, c.first, c.second);
         if (r.code) { why = r.msg; why_code = r.code; continue; }
-        build_segments(P, Lmax);
+        build_segplan(P, P.seg[0], 32);
+        build_segplan(P, P.seg[1], 64);
         // self-check: residual of the equilibrated system with 4 random RHS
         const int nb = 4;
         std::vector<double> b((size_t)n * nb), x;

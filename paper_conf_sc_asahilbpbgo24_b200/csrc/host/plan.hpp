@@ -1,12 +1,12 @@
 // plan.hpp -- host-side "create" step of the spline builder: collocation
-// matrix, Schur split, one-time factorisation, COO corners and the segment
-// coupling data of the in-CTA parallel recurrence.
+// matrix, Schur split, one-time factorisation, sparse corner blocks and the
+// segment coupling data of the in-CTA parallel recurrences.
 //
 // "the factorization is only done once at
 // initialization ... we take advantage of existing CPU libraries to
 // factorize the matrix and copy the result to the device".  There is no
-// LAPACK on the target box, so the banded factorisations (pttrf / pbtrf /
-// gbtrf-without-interchanges, getrf for delta') are written here.
+// LAPACK on the target box, so the banded factorisations (pttrf / pbtrf-like
+// LDL^T, gbtrf without interchanges, getrf for delta') are written here.
 #pragma once
 #include <cstdint>
 #include <string>
@@ -17,13 +17,23 @@ namespace sb {
 enum Bc { PERIODIC = 0, GREVILLE = 1, HERMITE = 2 };
 enum QType { Q_PTTRS = 0, Q_PBTRS = 1, Q_GBTRS = 2 };
 
-constexpr int KMAX_BAND = 4;    // largest Q half-band the kernels are built for
-constexpr int KMAX_DELTA = 32;  // largest delta' order
-constexpr double BETA_DROP = 1e-14;  // keep |beta| > 1e-14 (DESIGN R4)
+constexpr int KMAX_BAND = 4;          // largest Q half-band the kernels are built for
+constexpr int KMAX_DELTA = 32;        // largest delta' order
+constexpr double CORNER_DROP = 1e-14; // keep |beta|, |Lambda| > 1e-14 (DESIGN R4)
 
 struct SparseRow {
     std::vector<int> col;
     std::vector<double> val;
+};
+
+// segment partition of the padded Q recurrences for one register segment
+// length L: S segments of exactly L rows, Q padded with
+// identity rows to nQp = S*L.
+struct SegPlan {
+    int L = 0, S = 0, nQp = 0;
+    int carry_f = 0, carry_b = 0;  // predecessor segments in the carry walks
+    std::vector<double> G;         // S*K*K forward transfer  G_t[j][m]
+    std::vector<double> H;         // S*K*K backward transfer H_t[j][m]
 };
 
 struct Plan {
@@ -38,36 +48,23 @@ struct Plan {
     int kl = 0, ku = 0, K = 1;      // Q band, kernel band (max, >=1)
     int qtype = Q_GBTRS;
     double growth = 0.0;
-    // ---- factors of Q in Q-local indices (forward unit-lower L, backward
-    // x_i = y_i*dinv_i - sum_m up_{i,m} x_{i+m})
+    // ---- factors of Q, Q-local indices (forward unit-lower L, backward
+    //      x_i = y_i*dinv_i - sum_m up_{i,m} x_{i+m})
     std::vector<double> Lb;         // nQ*K : Lb[i*K+m-1] = L(i, i-m)
     std::vector<double> Ub;         // nQ*K : Ub[i*K+m-1] = U(i, i+m)/U(i,i)
     std::vector<double> dinv;       // nQ
-    // ---- corners
-    std::vector<double> beta_full;  // nQ*k, beta = Q^{-1} gamma (Eq. 4)
-    std::vector<int> lam_r, lam_c;  std::vector<double> lam_v;   // lambda COO
-    std::vector<int> beta_r, beta_c; std::vector<double> beta_v; // beta COO (thresholded)
+    // ---- corners (Eq. 4 and its transposed twin)
+    std::vector<int> lam_r, lam_c;   std::vector<double> lam_v;    // lambda COO (delta row, Q col)
+    std::vector<int> gam_r, gam_c;   std::vector<double> gam_v;    // gamma COO (Q row, delta col), sorted by row
+    std::vector<int> beta_r, beta_c; std::vector<double> beta_v;   // beta = Q^-1 gamma, thresholded COO
+    std::vector<int> Lam_ptr, Lam_c; std::vector<double> Lam_v;    // Lambda = lambda Q^-1, thresholded CSR by delta row
     std::vector<double> dprime;     // k*k delta' = delta - lambda beta
     std::vector<double> dlu;        // k*k LU of delta' (getrf, partial pivoting)
     std::vector<int> dpiv;          // k
-    // ---- in-CTA segments of the Q recurrences
-    int Lmax = 32, S = 1, seg_base = 0, seg_rem = 0, Lseg = 0;
-    std::vector<double> gspk;       // nQ*K forward spikes
-    std::vector<double> hspk;       // nQ*K backward spikes
-    int carry_f = 0, carry_b = 0;
-    // ---- head / tail windows holding every lambda column and beta row
-    int Wh = 0, Wt = 0;
-
-    int seg_start(int s) const { return s * seg_base + (s < seg_rem ? s : seg_rem); }
-    int seg_len(int s) const { return seg_base + (s < seg_rem ? 1 : 0); }
-    int win_slot(int qrow) const {  // -1 if outside the windows
-        if (qrow < Wh) return qrow;
-        if (qrow >= nQ - Wt) return Wh + (qrow - (nQ - Wt));
-        return -1;
-    }
+    // ---- segment plans: [0] fp64 kernels (L=32), [1] fp32 kernels (L=64)
+    SegPlan seg[2];
 };
 
-// status codes mirror include/spline_builder.h
 struct Status {
     int code = 0;
     std::string msg;
@@ -75,11 +72,10 @@ struct Status {
 
 // Build the spline space, the (equilibrated) collocation matrix, choose the
 // split, factor, compute corners and segment data.  split_lo/hi = -1: default.
-Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi,
-                  int Lmax);
+Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi);
 
-// Algorithm 1 on the CPU with the plan's factors (serial, fp64): reference
-// used by create's self-check and exported for tests.
+// Algorithm 1 on the CPU with the plan's factors (serial, fp64), in the same
+// order as the kernels (Lambda / gamma form).  Used by create's self-check.
 void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, int64_t pstride);
 
 }  // namespace sb

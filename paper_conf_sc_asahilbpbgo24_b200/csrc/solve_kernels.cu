@@ -1,26 +1,30 @@
-// solve_kernels.cu -- fused sm_100a kernels of the batched spline solve.
+// solve_kernels.cu -- fused sm_100a kernel of the batched spline solve.
 //
-// One launch runs the whole of Algorithm 1 for every
-// right-hand side, the B200 counterpart of the paper's fused
-// "SerialPttrs_Spmv" kernel (Listing 6):
-//   step 2  Q x0' = b0       banded forward/backward recurrences (pttrs /
-//                            pbtrs / gbtrs, Listing 1, Table I)
-//   step 3  delta' x1 = b1 - lambda x0'   COO spmv + getrs
-//   step 4  x0 = x0' - beta x1            COO spmv
+// One launch runs the whole Schur-complement chain (Eq. 3-6,
+// Algorithm 1) for every right-hand side -- the B200 counterpart of
+// the paper's fused "SerialPttrs_Spmv" kernel (Listing 6).  The
+// block LU is applied in its transposed form A = [[I,0],[Lambda,I]] [[Q,gamma],[0,delta']]
+// with Lambda = lambda Q^{-1} (R6), which gives the same x:
+//   corner  x1 = delta'^{-1} (b1 - Lambda b0)   COO/CSR spmv + getrs
+//   gamma   b0 <- b0 - gamma x1                  COO spmv (transposed)
+//   Q       x0 = Q^{-1} b0                        banded LDL^T / LU recurrences
+//                                                 (pttrs / pbtrs / gbtrs, Listing 1, Table I)
+// so the corner work reads only input rows of the tile already in shared
+// memory and the Q solution goes straight from registers to HBM.
 //
-// B200 design, unlike the paper's one-thread-per-RHS
-// walk over HBM (which re-reads every element):
-//  * a CTA owns a tile of R right-hand sides; the tile is staged in shared
-//    memory by TMA (cp.async.bulk.tensor, mbarrier-tracked) while the previous
-//    tile is being solved, so HBM sees exactly one read and one write of each
-//    element;
-//  * thread (r, s) holds segment s of the Q rows of RHS r in registers; the
-//    recurrences run locally with zero inflow and are made exact by the
-//    precomputed spike vectors of the segment partition (truncated SPIKE):
-//    carries go through shared memory, the fix-up is fused into the next sweep;
-//  * factor bands, spikes, corner COO and delta' LU are staged once per CTA
-//    in shared memory and read as warp broadcasts;
-//  * the corner steps touch only the head/tail windows of Q.
+// B200 mapping:
+//  * persistent CTA (one per SM) owns a tile of R right-hand sides x all n
+//    rows; the next tile is fetched by TMA (cp.async.bulk.tensor 2-D,
+//    mbarrier complete_tx) while the current one is solved -> each element is
+//    read once and written once (16 B / element in fp64);
+//  * thread (r, s) keeps rows [s*L, s*L+L) of RHS r in registers; the
+//    recurrences run locally with zero inflow, then the exact inflow /
+//    outflow ("carries") is obtained from the neighbours' end states through
+//    shared memory and the precomputed segment transfer matrices, and added
+//    back by a correction chain (SPIKE-style) -- exact, no overlap, no re-read;
+//  * Q is padded with identity rows to S*L so the sweeps carry no predicates;
+//  * factors, transfer matrices and corner data are staged once per CTA in
+//    shared memory and read as broadcasts.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
@@ -41,8 +45,8 @@ struct KParams {
     int64_t batch, bstride, pstride;
     int ntiles, nbox, boxr;
     // dynamic shared memory offsets (bytes)
-    int off_buf, off_fwd, off_bwd, off_fend, off_bbeg, off_win, off_b1, off_x1, off_betaW, off_lamv, off_lamr,
-        off_lams, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, smem_total;
+    int off_buf, off_L, off_U, off_dinv, off_G, off_H, off_fend, off_bbeg, off_x1, off_lamptr, off_lamc, off_lamv,
+        off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, smem_total;
 };
 
 // ------------------------------------------------------------- PTX helpers
@@ -79,39 +83,45 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
 }
 
 template <typename T>
-__device__ __forceinline__ void stg_stream(T *p, T v) {
-    __stcs(p, v);  // streaming store: written once, not re-read by this kernel
+__device__ __forceinline__ void copy_words(T *dst, const T *src, int count, int tid, int nthreads) {
+    for (int i = tid; i < count; i += nthreads) dst[i] = src[i];
 }
 
 // ------------------------------------------------------------------ kernel
-template <typename T, int K, int LMAX, int R, int LOADER>
+template <typename T, int K, int L, int R, int LOADER>
 __global__ void __launch_bounds__(512, 1)
     sb_solve_kernel(const __grid_constant__ KParams p, const __grid_constant__ CUtensorMap tmap) {
-    using C = T;  // compute in the storage precision (fp64 -> fp64, fp32 -> fp32)
-    constexpr int CI = sizeof(C) == 8 ? 0 : 1;
-    constexpr int FS = 2 * K;      // forward record: L(i,i-1..i-K), g^(1..K)_i
-    constexpr int BS = 2 * K + 2;  // backward record: dinv_i, U'(i,1..K), h^(1..K)_i, pad
+    using C = T;  // compute in the storage precision
+    constexpr int CI = sizeof(T) == 8 ? 0 : 1;
+    constexpr int CP = 32 / R;  // corner lanes per RHS in warp 0
+    static_assert(L % 2 == 0, "segment length must be even");
     extern __shared__ __align__(1024) unsigned char smem[];
     const DevPlan &P = p.P;
+    const DevSeg &G = P.seg[CI];
 
     const int tid = threadIdx.x;
+    const int nthreads = blockDim.x;
     const int r = tid % R;
     const int s = tid / R;
-    const int S = P.S, nQ = P.nQ, k = P.k, Wh = P.Wh, Wt = P.Wt, W = P.Wh + P.Wt;
-    const int a = s * P.seg_base + min(s, P.seg_rem);
-    const int len = P.seg_base + (s < P.seg_rem ? 1 : 0);
+    const int S = G.S, nQ = P.nQ, k = P.k, nQpa = P.nQpa;
+    const int a = s * L;
+    const bool full = a + L <= nQ;  // segment has no padding rows
 
-    C *sfwd = reinterpret_cast<C *>(smem + p.off_fwd);
-    C *sbwd = reinterpret_cast<C *>(smem + p.off_bwd);
+    C *sL = reinterpret_cast<C *>(smem + p.off_L);
+    C *sU = reinterpret_cast<C *>(smem + p.off_U);
+    C *sdinv = reinterpret_cast<C *>(smem + p.off_dinv);
+    C *sG = reinterpret_cast<C *>(smem + p.off_G);
+    C *sH = reinterpret_cast<C *>(smem + p.off_H);
     C *sfend = reinterpret_cast<C *>(smem + p.off_fend);
     C *sbbeg = reinterpret_cast<C *>(smem + p.off_bbeg);
-    C *swin = reinterpret_cast<C *>(smem + p.off_win);
-    C *sb1 = reinterpret_cast<C *>(smem + p.off_b1);
     C *sx1 = reinterpret_cast<C *>(smem + p.off_x1);
-    C *sbeta = reinterpret_cast<C *>(smem + p.off_betaW);
+    int *slamptr = reinterpret_cast<int *>(smem + p.off_lamptr);
+    int *slamc = reinterpret_cast<int *>(smem + p.off_lamc);
     C *slamv = reinterpret_cast<C *>(smem + p.off_lamv);
-    int *slamr = reinterpret_cast<int *>(smem + p.off_lamr);
-    int *slams = reinterpret_cast<int *>(smem + p.off_lams);
+    int *sgamr = reinterpret_cast<int *>(smem + p.off_gamr);
+    int *sgamc = reinterpret_cast<int *>(smem + p.off_gamc);
+    C *sgamv = reinterpret_cast<C *>(smem + p.off_gamv);
+    int *sgptr = reinterpret_cast<int *>(smem + p.off_gptr);
     C *sdlu = reinterpret_cast<C *>(smem + p.off_dlu);
     int *sdpiv = reinterpret_cast<int *>(smem + p.off_dpiv);
     C *sdscale = reinterpret_cast<C *>(smem + p.off_dscale);
@@ -119,229 +129,227 @@ __global__ void __launch_bounds__(512, 1)
     uint64_t *mbar = reinterpret_cast<uint64_t *>(smem + p.off_mbar);
     T *buf = reinterpret_cast<T *>(smem + p.off_buf);
 
-    const int nthreads = blockDim.x;
     int tile = blockIdx.x;
+    const uint32_t tile_bytes = (uint32_t)(p.nbox * p.boxr * R * sizeof(T));
 
-    // kick off the first tile before staging the constants (overlap)
+    // first tile in flight while the constants are staged
     if (LOADER == LOAD_TMA && tid == 0) {
         prefetch_tmap(&tmap);
         mbar_init(mbar, 1);
         fence_mbar_init();
         if (tile < p.ntiles) {
-            mbar_arrive_expect_tx(mbar, (uint32_t)(p.nbox * p.boxr * R * sizeof(T)));
+            mbar_arrive_expect_tx(mbar, tile_bytes);
             for (int b = 0; b < p.nbox; ++b) tma_load_2d(buf + (size_t)b * p.boxr * R, &tmap, mbar, tile * R, b * p.boxr);
         }
     }
-    // stage constants (factor records, corners) once per CTA
     {
-        const float4 *src = reinterpret_cast<const float4 *>(P.fwd[CI]);
-        float4 *dst = reinterpret_cast<float4 *>(sfwd);
-        const int nv = (int)(((size_t)nQ * FS * sizeof(C) + 15) / 16);  // sections padded to 16 B
-        for (int i = tid; i < nv; i += nthreads) dst[i] = src[i];
-        src = reinterpret_cast<const float4 *>(P.bwd[CI]);
-        dst = reinterpret_cast<float4 *>(sbwd);
-        const int nb = (int)(((size_t)nQ * BS * sizeof(C) + 15) / 16);
-        for (int i = tid; i < nb; i += nthreads) dst[i] = src[i];
-        const C *bw = reinterpret_cast<const C *>(P.betaW[CI]);
-        for (int i = tid; i < W * k; i += nthreads) sbeta[i] = bw[i];
-        const C *lv = reinterpret_cast<const C *>(P.lam_v[CI]);
-        for (int i = tid; i < P.nlam; i += nthreads) {
-            slamv[i] = lv[i];
-            slamr[i] = P.lam_r[i];
-            slams[i] = P.lam_slot[i];
-        }
-        const C *dl = reinterpret_cast<const C *>(P.dlu[CI]);
-        for (int i = tid; i < k * k; i += nthreads) sdlu[i] = dl[i];
-        const C *ds = reinterpret_cast<const C *>(P.dscale[CI]);
-        for (int i = tid; i < k; i += nthreads) {
-            sdpiv[i] = P.dpiv[i];
-            sdscale[i] = ds[i];
-            sdrow[i] = P.drow[i];
-        }
+        const int nrec = K * nQpa;
+        copy_words(sL, reinterpret_cast<const C *>(P.Lr[CI]), nrec, tid, nthreads);
+        copy_words(sU, reinterpret_cast<const C *>(P.Ur[CI]), nrec, tid, nthreads);
+        copy_words(sdinv, reinterpret_cast<const C *>(P.dinv[CI]), nQpa, tid, nthreads);
+        copy_words(sG, reinterpret_cast<const C *>(G.G), S * K * K, tid, nthreads);
+        copy_words(sH, reinterpret_cast<const C *>(G.H), S * K * K, tid, nthreads);
+        copy_words(slamptr, P.lam_ptr, k + 1, tid, nthreads);
+        copy_words(slamc, P.lam_c, P.lam_nnz, tid, nthreads);
+        copy_words(slamv, reinterpret_cast<const C *>(P.lam_v[CI]), P.lam_nnz, tid, nthreads);
+        copy_words(sgamr, P.gam_r, P.gam_nnz, tid, nthreads);
+        copy_words(sgamc, P.gam_c, P.gam_nnz, tid, nthreads);
+        copy_words(sgamv, reinterpret_cast<const C *>(P.gam_v[CI]), P.gam_nnz, tid, nthreads);
+        copy_words(sgptr, G.gptr, S + 1, tid, nthreads);
+        copy_words(sdlu, reinterpret_cast<const C *>(P.dlu[CI]), k * k, tid, nthreads);
+        copy_words(sdpiv, P.dpiv, k, tid, nthreads);
+        copy_words(sdscale, reinterpret_cast<const C *>(P.dscale[CI]), k, tid, nthreads);
+        copy_words(sdrow, P.drow, k, tid, nthreads);
     }
     __syncthreads();
 
     T *gout = reinterpret_cast<T *>(p.rhs);
+    const int64_t ps = p.pstride;
     uint32_t phase = 0;
     for (; tile < p.ntiles; tile += gridDim.x) {
         const int64_t col = (int64_t)tile * R + r;
         const bool live = col < p.batch;
         T *gcol = gout + col * p.bstride;
-        C v[LMAX];
-        // ---------------------------------------------------------- load
         if (LOADER == LOAD_TMA) {
             mbar_wait(mbar, phase);
             phase ^= 1u;
-            const T *brow = buf + (size_t)(P.s_lo + a) * R + r;
-#pragma unroll
-            for (int i = 0; i < LMAX; ++i)
-                if (i < len) v[i] = (C)brow[(size_t)i * R];
-            if (s == 0)
-                for (int d = 0; d < k; ++d) sb1[r * k + d] = (C)buf[(size_t)sdrow[d] * R + r] * sdscale[d];
-            __syncthreads();  // B1: tile buffer consumed -> refill it with the next tile
-            if (tid == 0 && tile + (int)gridDim.x < p.ntiles) {
-                const int nt = tile + gridDim.x;
-                mbar_arrive_expect_tx(mbar, (uint32_t)(p.nbox * p.boxr * R * sizeof(T)));
-                for (int b = 0; b < p.nbox; ++b)
-                    tma_load_2d(buf + (size_t)b * p.boxr * R, &tmap, mbar, nt * R, b * p.boxr);
-            }
-        } else {
-            const T *gsrc = gcol + (int64_t)(P.s_lo + a) * p.pstride;
-#pragma unroll
-            for (int i = 0; i < LMAX; ++i)
-                if (i < len) v[i] = live ? (C)__ldcs(gsrc + (int64_t)i * p.pstride) : C(0);
-            if (s == 0)
-                for (int d = 0; d < k; ++d)
-                    sb1[r * k + d] = live ? (C)gcol[(int64_t)sdrow[d] * p.pstride] * sdscale[d] : C(0);
         }
-        // ------------------------------- step 2a: local forward sweep (L y = b)
+        // ---------- corner: x1 = delta'^{-1} (s1*b1 - Lambda b0), warp 0 (CP lanes per RHS)
+        if (tid < 32 && k > 0) {
+            // CTAs with a single segment have only R (< 32) threads: one part
+            const int cp = min(CP, nthreads / R);
+            const int part = tid / R, rr = tid % R;
+            const int64_t ccol = (int64_t)tile * R + rr;
+            const bool clive = ccol < p.batch;
+            const T *ccolp = gout + ccol * p.bstride;
+            auto ldb = [&](int row) -> C {
+                if (LOADER == LOAD_TMA) return (C)buf[(size_t)row * R + rr];
+                return clive ? (C)ccolp[(int64_t)row * ps] : C(0);
+            };
+            for (int d = 0; d < k; ++d) {
+                C acc = part == 0 ? ldb(sdrow[d]) * sdscale[d] : C(0);
+                for (int e = slamptr[d] + part; e < slamptr[d + 1]; e += cp)
+                    acc = fma(-slamv[e], ldb(P.s_lo + slamc[e]), acc);
+                if (cp > 1) {
+#pragma unroll
+                    for (int off = R; off < 32; off *= 2) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+                }
+                if (part == 0) sx1[rr * k + d] = acc;
+            }
+            if (part == 0) {
+                C *x1 = sx1 + rr * k;
+                for (int d = 0; d < k; ++d) {
+                    const int pv = sdpiv[d];
+                    if (pv != d) { C t = x1[d]; x1[d] = x1[pv]; x1[pv] = t; }
+                }
+                for (int i = 1; i < k; ++i)
+                    for (int j = 0; j < i; ++j) x1[i] = fma(-sdlu[i * k + j], x1[j], x1[i]);
+                for (int i = k - 1; i >= 0; --i) {
+                    C acc = x1[i];
+                    for (int j = i + 1; j < k; ++j) acc = fma(-sdlu[i * k + j], x1[j], acc);
+                    x1[i] = acc / sdlu[i * k + i];
+                }
+                if (clive)
+                    for (int d = 0; d < k; ++d) __stcs(gout + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
+            }
+        }
+        // ---------- own segment of b0 into registers
+        C v[L];
+        {
+            if (LOADER == LOAD_TMA) {
+                const T *src = buf + (size_t)(P.s_lo + a) * R + r;
+                if (full) {
+#pragma unroll
+                    for (int i = 0; i < L; ++i) v[i] = (C)src[(size_t)i * R];
+                } else {
+#pragma unroll
+                    for (int i = 0; i < L; ++i) v[i] = (a + i < nQ) ? (C)src[(size_t)i * R] : C(0);
+                }
+            } else {
+                const T *src = gcol + (int64_t)(P.s_lo + a) * ps;
+                if (full && live) {
+#pragma unroll
+                    for (int i = 0; i < L; ++i) v[i] = (C)__ldcs(src + (int64_t)i * ps);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < L; ++i) v[i] = (live && a + i < nQ) ? (C)__ldcs(src + (int64_t)i * ps) : C(0);
+                }
+            }
+        }
+        __syncthreads();  // B1: tile buffer consumed, x1 published
+        if (LOADER == LOAD_TMA && tid == 0 && tile + (int)gridDim.x < p.ntiles) {
+            const int nt = tile + gridDim.x;
+            mbar_arrive_expect_tx(mbar, tile_bytes);
+            for (int b = 0; b < p.nbox; ++b) tma_load_2d(buf + (size_t)b * p.boxr * R, &tmap, mbar, nt * R, b * p.boxr);
+        }
+        // ---------- b0 -= gamma x1 on this segment's gamma rows
+        for (int e = sgptr[s]; e < sgptr[s + 1]; ++e) {
+            const int i = sgamr[e] - a;
+            const C dv = sgamv[e] * sx1[r * k + sgamc[e]];
+#pragma unroll
+            for (int j = 0; j < L; ++j)
+                if (j == i) v[j] -= dv;
+        }
+        // ---------- local forward sweep, zero inflow:  y_i = b_i - sum_m L(i,i-m) y_{i-m}
         C st[K];
 #pragma unroll
         for (int m = 0; m < K; ++m) st[m] = C(0);
-        {
-            const C *f = sfwd + (size_t)a * FS;
 #pragma unroll
-            for (int i = 0; i < LMAX; ++i) {
-                if (i < len) {
-                    C acc = v[i];
+        for (int i = 0; i < L; ++i) {
+            C acc = v[i];
 #pragma unroll
-                    for (int m = 0; m < K; ++m) acc = fma(-f[i * FS + m], st[m], acc);
+            for (int m = 0; m < K; ++m) acc = fma(-sL[m * nQpa + a + i], st[m], acc);
 #pragma unroll
-                    for (int m = K - 1; m > 0; --m) st[m] = st[m - 1];
-                    st[0] = acc;
-                    v[i] = acc;
-                }
-            }
+            for (int m = K - 1; m > 0; --m) st[m] = st[m - 1];
+            st[0] = acc;
+            v[i] = acc;
         }
 #pragma unroll
         for (int j = 0; j < K; ++j) sfend[(s * R + r) * K + j] = st[j];
         __syncthreads();  // B2
-        // forward carry: true y at rows a-1..a-K (walk over predecessor segments)
-        C cin[K];
-#pragma unroll
-        for (int m = 0; m < K; ++m) cin[m] = C(0);
+        // ---------- forward carry (true y at rows a-1..a-K) and correction chain
         if (s > 0) {
-            const int t0 = max(0, s - P.carry_f);
-            for (int t = t0; t < s; ++t) {
-                const int end = t * P.seg_base + min(t, P.seg_rem) + P.seg_base + (t < P.seg_rem ? 1 : 0);
+            C cin[K];
+#pragma unroll
+            for (int m = 0; m < K; ++m) cin[m] = C(0);
+            for (int t = max(0, s - G.carry_f); t < s; ++t) {
                 C nw[K];
 #pragma unroll
                 for (int j = 0; j < K; ++j) {
                     C acc = sfend[(t * R + r) * K + j];
-                    const C *g = sfwd + (size_t)(end - 1 - j) * FS + K;
 #pragma unroll
-                    for (int m = 0; m < K; ++m) acc = fma(g[m], cin[m], acc);
+                    for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m], acc);
                     nw[j] = acc;
                 }
 #pragma unroll
                 for (int j = 0; j < K; ++j) cin[j] = nw[j];
             }
+            // c_i = -sum_m L(i,i-m) c_{i-m}, c_{a-m} = cin ;  y_i += c_i
+#pragma unroll
+            for (int i = 0; i < L; ++i) {
+                C c = C(0);
+#pragma unroll
+                for (int m = 0; m < K; ++m) c = fma(-sL[m * nQpa + a + i], cin[m], c);
+#pragma unroll
+                for (int m = K - 1; m > 0; --m) cin[m] = cin[m - 1];
+                cin[0] = c;
+                v[i] += c;
+            }
         }
-        // ---------- step 2b: forward fix-up fused into the local backward sweep
+        // ---------- local backward sweep, zero outflow: x_i = y_i dinv_i - sum_m U'(i,m) x_{i+m}
         C st2[K];
 #pragma unroll
         for (int m = 0; m < K; ++m) st2[m] = C(0);
-        {
-            const C *f = sfwd + (size_t)a * FS;
-            const C *b = sbwd + (size_t)a * BS;
-            const bool fix = s > 0;
 #pragma unroll
-            for (int i = LMAX - 1; i >= 0; --i) {
-                if (i < len) {
-                    C y = v[i];
-                    if (fix) {
+        for (int i = L - 1; i >= 0; --i) {
+            C acc = v[i] * sdinv[a + i];
 #pragma unroll
-                        for (int m = 0; m < K; ++m) y = fma(f[i * FS + K + m], cin[m], y);
-                    }
-                    C acc = y * b[i * BS];
+            for (int m = 0; m < K; ++m) acc = fma(-sU[m * nQpa + a + i], st2[m], acc);
 #pragma unroll
-                    for (int m = 0; m < K; ++m) acc = fma(-b[i * BS + 1 + m], st2[m], acc);
-#pragma unroll
-                    for (int m = K - 1; m > 0; --m) st2[m] = st2[m - 1];
-                    st2[0] = acc;
-                    v[i] = acc;
-                }
-            }
+            for (int m = K - 1; m > 0; --m) st2[m] = st2[m - 1];
+            st2[0] = acc;
+            v[i] = acc;
         }
 #pragma unroll
         for (int j = 0; j < K; ++j) sbbeg[(s * R + r) * K + j] = st2[j];
         __syncthreads();  // B3
-        C cout[K];
-#pragma unroll
-        for (int m = 0; m < K; ++m) cout[m] = C(0);
+        // ---------- backward carry (true x at rows a+L..a+L+K-1), correction chain, store
+        T *dst = gcol + (int64_t)(P.s_lo + a) * ps;
         if (s < S - 1) {
-            const int t0 = min(S - 1, s + P.carry_b);
-            for (int t = t0; t > s; --t) {
-                const int at = t * P.seg_base + min(t, P.seg_rem);
+            C co[K];
+#pragma unroll
+            for (int m = 0; m < K; ++m) co[m] = C(0);
+            for (int t = min(S - 1, s + G.carry_b); t > s; --t) {
                 C nw[K];
 #pragma unroll
                 for (int j = 0; j < K; ++j) {
                     C acc = sbbeg[(t * R + r) * K + j];
-                    const C *h = sbwd + (size_t)(at + j) * BS + 1 + K;
 #pragma unroll
-                    for (int m = 0; m < K; ++m) acc = fma(h[m], cout[m], acc);
+                    for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m], acc);
                     nw[j] = acc;
                 }
 #pragma unroll
-                for (int j = 0; j < K; ++j) cout[j] = nw[j];
+                for (int j = 0; j < K; ++j) co[j] = nw[j];
+            }
+#pragma unroll
+            for (int i = L - 1; i >= 0; --i) {
+                C c = C(0);
+#pragma unroll
+                for (int m = 0; m < K; ++m) c = fma(-sU[m * nQpa + a + i], co[m], c);
+#pragma unroll
+                for (int m = K - 1; m > 0; --m) co[m] = co[m - 1];
+                co[0] = c;
+                v[i] += c;
             }
         }
-        // backward fix-up -> x0'; window rows go to smem, the rest straight to HBM
-        const bool inwin = (a < Wh) || (a + len > nQ - Wt);
-        {
-            const C *b = sbwd + (size_t)a * BS;
-            const bool fix = s < S - 1;
-            T *grow = gcol + (int64_t)(P.s_lo + a) * p.pstride;
+        if (live) {
+            if (full) {
 #pragma unroll
-            for (int i = 0; i < LMAX; ++i) {
-                if (i < len) {
-                    if (fix) {
+                for (int i = 0; i < L; ++i) __stcs(dst + (int64_t)i * ps, (T)v[i]);
+            } else {
 #pragma unroll
-                        for (int m = 0; m < K; ++m) v[i] = fma(b[i * BS + 1 + K + m], cout[m], v[i]);
-                    }
-                    const int q = a + i;
-                    const int slot = q < Wh ? q : (q >= nQ - Wt ? Wh + q - (nQ - Wt) : -1);
-                    if (slot >= 0) swin[r * W + slot] = v[i];
-                    else if (live) stg_stream(grow + (int64_t)i * p.pstride, (T)v[i]);
-                }
-            }
-        }
-        __syncthreads();  // B4
-        // ------------- step 3: x1 = delta'^{-1} (b1 - lambda x0')  (one thread per RHS)
-        if (s == 0 && k > 0) {
-            C *x1 = sx1 + r * k;
-            for (int d = 0; d < k; ++d) x1[d] = sb1[r * k + d];
-            for (int e = 0; e < P.nlam; ++e) x1[slamr[e]] = fma(-slamv[e], swin[r * W + slams[e]], x1[slamr[e]]);
-            for (int d = 0; d < k; ++d) {
-                const int pv = sdpiv[d];
-                if (pv != d) { C t = x1[d]; x1[d] = x1[pv]; x1[pv] = t; }
-            }
-            for (int i = 1; i < k; ++i)
-                for (int j = 0; j < i; ++j) x1[i] = fma(-sdlu[i * k + j], x1[j], x1[i]);
-            for (int i = k - 1; i >= 0; --i) {
-                C acc = x1[i];
-                for (int j = i + 1; j < k; ++j) acc = fma(-sdlu[i * k + j], x1[j], acc);
-                x1[i] = acc / sdlu[i * k + i];
-            }
-            if (live)
-                for (int d = 0; d < k; ++d) stg_stream(gcol + (int64_t)sdrow[d] * p.pstride, (T)x1[d]);
-        }
-        __syncthreads();  // B5
-        // ------------------------------------ step 4: x0 = x0' - beta x1 (windows)
-        if (inwin) {
-            const C *x1 = sx1 + r * k;
-            T *grow = gcol + (int64_t)(P.s_lo + a) * p.pstride;
-#pragma unroll
-            for (int i = 0; i < LMAX; ++i) {
-                if (i < len) {
-                    const int q = a + i;
-                    const int slot = q < Wh ? q : (q >= nQ - Wt ? Wh + q - (nQ - Wt) : -1);
-                    if (slot >= 0) {
-                        C acc = v[i];
-                        for (int c = 0; c < k; ++c) acc = fma(-sbeta[slot * k + c], x1[c], acc);
-                        if (live) stg_stream(grow + (int64_t)i * p.pstride, (T)acc);
-                    }
-                }
+                for (int i = 0; i < L; ++i)
+                    if (a + i < nQ) __stcs(dst + (int64_t)i * ps, (T)v[i]);
             }
         }
     }
@@ -350,7 +358,6 @@ __global__ void __launch_bounds__(512, 1)
 // ------------------------------------------------------------------ host
 namespace {
 
-constexpr int LMAX = 32;
 constexpr int MAX_THREADS = 512;
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
@@ -369,9 +376,9 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
-template <typename T, int K, int R, int LOADER>
+template <typename T, int K, int L, int R, int LOADER>
 int launch_t(const KParams &kp, const CUtensorMap &tm, int grid, int threads, cudaStream_t st, char *err, int errlen) {
-    auto fn = sb_solve_kernel<T, K, LMAX, R, LOADER>;
+    auto fn = sb_solve_kernel<T, K, L, R, LOADER>;
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total);
     if (e != cudaSuccess) {
         snprintf(err, errlen, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
@@ -386,55 +393,68 @@ int launch_t(const KParams &kp, const CUtensorMap &tm, int grid, int threads, cu
     return 0;
 }
 
-template <typename T, int R, int LOADER>
+template <typename T, int L, int R, int LOADER>
 int dispatch_K(int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads, cudaStream_t st, char *err,
                int errlen) {
     switch (K) {
-        case 1: return launch_t<T, 1, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
-        case 2: return launch_t<T, 2, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
-        case 3: return launch_t<T, 3, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
-        case 4: return launch_t<T, 4, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
+        case 1: return launch_t<T, 1, L, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
+        case 2: return launch_t<T, 2, L, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
+        case 3: return launch_t<T, 3, L, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
+        case 4: return launch_t<T, 4, L, R, LOADER>(kp, tm, grid, threads, st, err, errlen);
     }
     snprintf(err, errlen, "unsupported band K=%d", K);
     return 5;
 }
 
-template <typename T>
-int dispatch(int R, int loader, int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads,
+// (dtype, R, loader) -> instantiation.  fp64: L=32, R in {16, 8};
+// fp32: L=64, R in {32, 16}.
+int dispatch(int dtype, int R, int loader, int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads,
              cudaStream_t st, char *err, int errlen) {
-    if (R == 16 && loader == LOAD_TMA) return dispatch_K<T, 16, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen);
-    if (R == 8 && loader == LOAD_TMA) return dispatch_K<T, 8, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen);
-    if (R == 16) return dispatch_K<T, 16, LOAD_DIRECT>(K, kp, tm, grid, threads, st, err, errlen);
-    if (R == 8) return dispatch_K<T, 8, LOAD_DIRECT>(K, kp, tm, grid, threads, st, err, errlen);
+    const bool tma = loader == LOAD_TMA;
+    if (dtype == 0) {
+        if (R == 16) return tma ? dispatch_K<double, 32, 16, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen)
+                                : dispatch_K<double, 32, 16, LOAD_DIRECT>(K, kp, tm, grid, threads, st, err, errlen);
+        if (R == 8) return tma ? dispatch_K<double, 32, 8, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen)
+                               : dispatch_K<double, 32, 8, LOAD_DIRECT>(K, kp, tm, grid, threads, st, err, errlen);
+    } else {
+        if (R == 32) return tma ? dispatch_K<float, 64, 32, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen)
+                                : dispatch_K<float, 64, 32, LOAD_DIRECT>(K, kp, tm, grid, threads, st, err, errlen);
+        if (R == 16) return tma ? dispatch_K<float, 64, 16, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen)
+                                : dispatch_K<float, 64, 16, LOAD_DIRECT>(K, kp, tm, grid, threads, st, err, errlen);
+    }
     snprintf(err, errlen, "unsupported tile width R=%d", R);
     return 5;
 }
 
-// lay out dynamic smem; returns total bytes
-int layout_smem(KParams &kp, const DevPlan &P, int R, size_t esz, bool with_buf, int nbox, int boxr) {
+int layout_smem(KParams &kp, const DevPlan &P, int R, size_t esz, bool with_buf, int nbox, int boxr, int S) {
     size_t o = 0;
     auto take = [&](size_t bytes, size_t al) {
         o = align_up(o, al);
         size_t r = o;
-        o += bytes;
+        o += align_up(bytes, 16);
         return (int)r;
     };
+    const int K = P.K, k = P.k;
     kp.off_buf = with_buf ? take((size_t)nbox * boxr * R * esz, 1024) : 0;
-    kp.off_fwd = take((size_t)P.nQ * P.fstride * esz, 16);
-    kp.off_bwd = take((size_t)P.nQ * P.bstride * esz, 16);
-    kp.off_fend = take((size_t)P.S * R * P.K * esz, 16);
-    kp.off_bbeg = take((size_t)P.S * R * P.K * esz, 16);
-    kp.off_win = take((size_t)R * (P.Wh + P.Wt) * esz, 16);
-    kp.off_b1 = take((size_t)R * P.k * esz, 16);
-    kp.off_x1 = take((size_t)R * P.k * esz, 16);
-    kp.off_betaW = take((size_t)(P.Wh + P.Wt) * P.k * esz, 16);
-    kp.off_lamv = take((size_t)P.nlam * esz, 16);
-    kp.off_lamr = take((size_t)P.nlam * 4, 16);
-    kp.off_lams = take((size_t)P.nlam * 4, 16);
-    kp.off_dlu = take((size_t)P.k * P.k * esz, 16);
-    kp.off_dpiv = take((size_t)P.k * 4, 16);
-    kp.off_dscale = take((size_t)P.k * esz, 16);
-    kp.off_drow = take((size_t)P.k * 4, 16);
+    kp.off_L = take((size_t)K * P.nQpa * esz, 16);
+    kp.off_U = take((size_t)K * P.nQpa * esz, 16);
+    kp.off_dinv = take((size_t)P.nQpa * esz, 16);
+    kp.off_G = take((size_t)S * K * K * esz, 16);
+    kp.off_H = take((size_t)S * K * K * esz, 16);
+    kp.off_fend = take((size_t)S * R * K * esz, 16);
+    kp.off_bbeg = take((size_t)S * R * K * esz, 16);
+    kp.off_x1 = take((size_t)R * k * esz, 16);
+    kp.off_lamptr = take((size_t)(k + 1) * 4, 16);
+    kp.off_lamc = take((size_t)P.lam_nnz * 4, 16);
+    kp.off_lamv = take((size_t)P.lam_nnz * esz, 16);
+    kp.off_gamr = take((size_t)P.gam_nnz * 4, 16);
+    kp.off_gamc = take((size_t)P.gam_nnz * 4, 16);
+    kp.off_gamv = take((size_t)P.gam_nnz * esz, 16);
+    kp.off_gptr = take((size_t)(S + 1) * 4, 16);
+    kp.off_dlu = take((size_t)k * k * esz, 16);
+    kp.off_dpiv = take((size_t)k * 4, 16);
+    kp.off_dscale = take((size_t)k * esz, 16);
+    kp.off_drow = take((size_t)k * 4, 16);
     kp.off_mbar = take(8, 8);
     kp.smem_total = (int)align_up(o, 16);
     return kp.smem_total;
@@ -442,14 +462,10 @@ int layout_smem(KParams &kp, const DevPlan &P, int R, size_t esz, bool with_buf,
 
 }  // namespace
 
-size_t const_smem_bytes(const DevPlan &P, int dtype) {
-    KParams kp{};
-    return (size_t)layout_smem(kp, P, 16, dtype == 0 ? 8 : 4, false, 0, 0);
-}
-
 int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, int errlen) {
     if (a.batch == 0) return 0;
     const size_t esz = a.dtype == 0 ? 8 : 4;
+    const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
     int dev = 0;
     cudaGetDevice(&dev);
     int max_smem = 0;
@@ -462,32 +478,38 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
     kp.bstride = a.bstride;
     kp.pstride = a.pstride;
 
-    // tile width R and loader: TMA for the batch-contiguous layout when the
-    // tensor-map constraints hold and the tile fits in shared memory
+    // TMA for the batch-contiguous layout when the tensor-map rules hold
+    // (16-B aligned base and row pitch) and the tile fits in shared memory.
     const bool contig = a.bstride == 1;
     const bool aligned = ((uintptr_t)a.rhs % 16 == 0) && ((a.pstride * (int64_t)esz) % 16 == 0);
     const int nbox = (P.n + 255) / 256;
     const int boxr = ((P.n + nbox - 1) / nbox + 7) / 8 * 8;
+    const int cands64[2] = {16, 8}, cands32[2] = {32, 16};
+    const int *cands = a.dtype == 0 ? cands64 : cands32;
     int R = 0, loader = LOAD_DIRECT;
-    CUtensorMap tm;
-    memset(&tm, 0, sizeof(tm));
-    for (int cand : {16, 8}) {
-        if (cand * P.S > MAX_THREADS) continue;
-        if (contig && aligned && a.batch >= cand && get_encode()) {
-            KParams t = kp;
-            if (layout_smem(t, P, cand, esz, true, nbox, boxr) <= max_smem) { R = cand; loader = LOAD_TMA; break; }
-        }
+    for (int ci = 0; ci < 2 && !R; ++ci) {
+        const int cand = cands[ci];
+        if (cand * G.S > MAX_THREADS) continue;
         KParams t = kp;
-        if (layout_smem(t, P, cand, esz, false, 0, 0) <= max_smem) { R = cand; loader = LOAD_DIRECT; break; }
+        if (contig && aligned && a.batch >= cand && get_encode() &&
+            layout_smem(t, P, cand, esz, true, nbox, boxr, G.S) <= max_smem) {
+            R = cand;
+            loader = LOAD_TMA;
+        } else if (layout_smem(t, P, cand, esz, false, 0, 0, G.S) <= max_smem) {
+            R = cand;
+            loader = LOAD_DIRECT;
+        }
     }
     if (!R) {
-        snprintf(err, errlen, "problem too large for the shared-memory kernel (n=%d, S=%d)", P.n, P.S);
+        snprintf(err, errlen, "problem too large for the shared-memory kernel (n=%d, segments=%d)", P.n, G.S);
         return 5;
     }
-    layout_smem(kp, P, R, esz, loader == LOAD_TMA, nbox, boxr);
+    layout_smem(kp, P, R, esz, loader == LOAD_TMA, nbox, boxr, G.S);
     kp.ntiles = (int)((a.batch + R - 1) / R);
     kp.nbox = nbox;
     kp.boxr = boxr;
+    CUtensorMap tm;
+    memset(&tm, 0, sizeof(tm));
     if (loader == LOAD_TMA) {
         cuuint64_t dims[2] = {(cuuint64_t)a.batch, (cuuint64_t)P.n};
         cuuint64_t strides[1] = {(cuuint64_t)(a.pstride * (int64_t)esz)};
@@ -502,10 +524,9 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
             return 3;
         }
     }
-    const int threads = R * P.S;
+    const int threads = R * G.S;
     const int grid = (int)std::min<int64_t>((int64_t)kp.ntiles, (int64_t)num_sms);
-    if (a.dtype == 0) return dispatch<double>(R, loader, P.K, kp, tm, grid, threads, a.stream, err, errlen);
-    return dispatch<float>(R, loader, P.K, kp, tm, grid, threads, a.stream, err, errlen);
+    return dispatch(a.dtype, R, loader, P.K, kp, tm, grid, threads, a.stream, err, errlen);
 }
 
 }  // namespace sb
