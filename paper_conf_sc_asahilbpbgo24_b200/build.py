@@ -22,8 +22,12 @@ SOURCES = [
     ("host/plan.cpp", "cxx"),
     ("capi.cpp", "cxx"),
     ("solve_kernels.cu", "cu"),
+    ("tile_f64.cu", "cu"),
+    ("tile_f32.cu", "cu"),
+    ("warp_f64.cu", "cu"),
+    ("warp_f32.cu", "cu"),
 ]
-HEADERS = ["host/plan.hpp", "device.hpp"]
+HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh"]
 
 
 def _newer(target: str, deps: list[str]) -> bool:
@@ -36,7 +40,7 @@ def _newer(target: str, deps: list[str]) -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "spline_builder.h")]
-    objs = []
+    objs, jobs = [], []
     for src, kind in SOURCES:
         path = os.path.join(CSRC, src)
         obj = os.path.join(BUILD, src.replace("/", "_") + ".o")
@@ -51,12 +55,20 @@ def build(force: bool = False, verbose: bool = False) -> str:
                    "--expt-relaxed-constexpr", "-c", path, "-o", obj]
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
+        jobs.append((cmd, obj, kind))
+
+    def run(job):
+        cmd, obj, kind = job
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"compile failed: {' '.join(cmd)}\n{r.stdout}\n{r.stderr}")
         if kind == "cu":
             with open(obj + ".ptxas.txt", "w") as f:
                 f.write(r.stderr)
+
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=max(1, min(len(jobs), os.cpu_count() or 4))) as ex:
+        list(ex.map(run, jobs))
     if force or _newer(LIB, objs):
         cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", LIB + ".tmp", *objs, "-lpthread", "-ldl", "-lrt"]
         r = subprocess.run(cmd, capture_output=True, text=True)

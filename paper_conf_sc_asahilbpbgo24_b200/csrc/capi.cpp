@@ -67,40 +67,50 @@ std::vector<C> conv(const std::vector<double> &v) {
 int upload(spline_builder *h) {
     const sb::Plan &P = h->plan;
     const int K = P.K, nQ = P.nQ, k = P.k;
-    // padded SoA factor arrays: stride nQpa covers both segment plans
-    const int nQpa = std::max(std::max(P.seg[0].nQp, P.seg[1].nQp), 2);
-    std::vector<double> Lr((size_t)K * nQpa, 0.0), Ur((size_t)K * nQpa, 0.0), dinv(nQpa, 1.0);
-    for (int i = 0; i < nQ; ++i) {
-        for (int m = 0; m < K; ++m) {
-            Lr[(size_t)m * nQpa + i] = P.Lb[(size_t)i * K + m];
-            Ur[(size_t)m * nQpa + i] = P.Ub[(size_t)i * K + m];
-        }
-        dinv[i] = P.dinv[i];
-    }
     std::vector<double> dscale(k);
     for (int d = 0; d < k; ++d) dscale[d] = P.rowscale[P.drow[d]];
-    // gamma entries of each segment (COO sorted by Q row)
-    std::vector<int> gptr[2];
-    for (int c = 0; c < 2; ++c) {
-        const sb::SegPlan &G = P.seg[c];
-        gptr[c].assign(G.S + 1, 0);
-        for (int s = 0, e = 0; s <= G.S; ++s) {
-            while (e < (int)P.gam_r.size() && P.gam_r[e] < s * G.L) ++e;
-            gptr[c][s] = e;
-        }
-        gptr[c][G.S] = (int)P.gam_r.size();
-    }
     Packer pk;
-    size_t oL[2], oU[2], oD[2], oLam[2], oGam[2], oDlu[2], oDs[2], oG[2], oH[2];
+    // per segment plan: factor arrays in the padded per-segment layout of device.hpp
+    struct SegOff { size_t L[2], U[2], D[2], G[2], H[2], gptr; int LP; };
+    SegOff so[3];
+    for (int g = 0; g < 3; ++g) {
+        const sb::SegPlan &G = P.seg[g];
+        // pitch: even (pair loads) and bank-staggered for the tile kernels (+2 fp64 / +4 fp32
+        // elements = 16 B); the warp kernel (odd L, lanes read distinct rows) needs no padding
+        const int LP = g == 0 ? G.L + 2 : (g == 1 ? G.L + 4 : G.L);
+        so[g].LP = LP;
+        const int S = G.S;
+        std::vector<double> Lr((size_t)K * S * LP, 0.0), Ur((size_t)K * S * LP, 0.0), dinv((size_t)S * LP, 1.0);
+        for (int s = 0; s < S; ++s)
+            for (int i = 0; i < G.L; ++i) {
+                const int row = s * G.L + i;
+                if (row >= nQ) continue;  // padding rows: identity
+                for (int m = 0; m < K; ++m) {
+                    Lr[((size_t)m * S + s) * LP + i] = P.Lb[(size_t)row * K + m];
+                    Ur[((size_t)m * S + s) * LP + i] = P.Ub[(size_t)row * K + m];
+                }
+                dinv[(size_t)s * LP + i] = P.dinv[row];
+            }
+        std::vector<int> gptr(S + 1, 0);
+        for (int s = 0, e = 0; s <= S; ++s) {
+            while (e < (int)P.gam_r.size() && P.gam_r[e] < s * G.L) ++e;
+            gptr[s] = e;
+        }
+        if (S > 0) gptr[S] = (int)P.gam_r.size();
+        so[g].L[0] = pk.addv(Lr); so[g].L[1] = pk.addv(conv<float>(Lr));
+        so[g].U[0] = pk.addv(Ur); so[g].U[1] = pk.addv(conv<float>(Ur));
+        so[g].D[0] = pk.addv(dinv); so[g].D[1] = pk.addv(conv<float>(dinv));
+        so[g].G[0] = pk.addv(G.G); so[g].G[1] = pk.addv(conv<float>(G.G));
+        so[g].H[0] = pk.addv(G.H); so[g].H[1] = pk.addv(conv<float>(G.H));
+        so[g].gptr = pk.addv(gptr);
+    }
+    size_t oLam[2], oGam[2], oDlu[2], oDs[2];
     for (int c = 0; c < 2; ++c) {
         auto put = [&](const std::vector<double> &v) { return c == 0 ? pk.addv(v) : pk.addv(conv<float>(v)); };
-        oL[c] = put(Lr); oU[c] = put(Ur); oD[c] = put(dinv);
         oLam[c] = put(P.Lam_v); oGam[c] = put(P.gam_v); oDlu[c] = put(P.dlu); oDs[c] = put(dscale);
-        oG[c] = put(P.seg[c].G); oH[c] = put(P.seg[c].H);
     }
     size_t o_lamptr = pk.addv(P.Lam_ptr), o_lamc = pk.addv(P.Lam_c), o_gamr = pk.addv(P.gam_r),
            o_gamc = pk.addv(P.gam_c), o_dpiv = pk.addv(P.dpiv), o_drow = pk.addv(P.drow);
-    size_t o_gptr[2] = {pk.addv(gptr[0]), pk.addv(gptr[1])};
     h->blob_bytes = std::max<size_t>(pk.bytes.size(), 16);
     cudaError_t e = cudaMalloc(&h->blob, h->blob_bytes);
     if (e != cudaSuccess) return fail(SB_NOMEM, std::string("cudaMalloc(blob): ") + cudaGetErrorString(e));
@@ -108,15 +118,20 @@ int upload(spline_builder *h) {
     if (e != cudaSuccess) return fail(SB_CUDA, std::string("cudaMemcpy(blob): ") + cudaGetErrorString(e));
     auto at = [&](size_t off) { return (const void *)((const unsigned char *)h->blob + off); };
     sb::DevPlan &d = h->dp;
-    d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K; d.nQpa = nQpa;
+    d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K;
     d.lam_nnz = (int)P.Lam_v.size(); d.gam_nnz = (int)P.gam_v.size();
     for (int c = 0; c < 2; ++c) {
-        d.Lr[c] = at(oL[c]); d.Ur[c] = at(oU[c]); d.dinv[c] = at(oD[c]);
         d.lam_v[c] = at(oLam[c]); d.gam_v[c] = at(oGam[c]); d.dlu[c] = at(oDlu[c]); d.dscale[c] = at(oDs[c]);
-        const sb::SegPlan &G = P.seg[c];
-        d.seg[c].L = G.L; d.seg[c].S = G.S; d.seg[c].nQp = G.nQp;
-        d.seg[c].carry_f = G.carry_f; d.seg[c].carry_b = G.carry_b;
-        d.seg[c].G = at(oG[c]); d.seg[c].H = at(oH[c]); d.seg[c].gptr = (const int *)at(o_gptr[c]);
+    }
+    for (int g = 0; g < 3; ++g) {
+        const sb::SegPlan &G = P.seg[g];
+        sb::DevSeg &ds = d.seg[g];
+        ds.L = G.L; ds.S = G.S; ds.LP = so[g].LP; ds.carry_f = G.carry_f; ds.carry_b = G.carry_b;
+        for (int c = 0; c < 2; ++c) {
+            ds.Lr[c] = at(so[g].L[c]); ds.Ur[c] = at(so[g].U[c]); ds.dinv[c] = at(so[g].D[c]);
+            ds.G[c] = at(so[g].G[c]); ds.H[c] = at(so[g].H[c]);
+        }
+        ds.gptr = (const int *)at(so[g].gptr);
     }
     d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
     d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);

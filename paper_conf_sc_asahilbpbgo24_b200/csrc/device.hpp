@@ -6,25 +6,29 @@
 
 namespace sb {
 
-// segment plan of one compute precision (register segment length L)
+// Segment plan of one kernel family: Q padded to S*L rows, split into S
+// register segments of L rows.  Factor arrays are stored per segment with a
+// padded pitch LP (bank-conflict-free broadcast reads, 16-B aligned pairs):
+//   L(a+i, a+i-1-m)  at Lr[(m*S + s)*LP + i]      (a = s*L)
+//   U'(a+i, a+i+1+m) at Ur[(m*S + s)*LP + i]
+//   dinv(a+i)        at dinv[s*LP + i]             (1 on padding rows)
+// Floating-point arrays exist in fp64 ([0]) and fp32 ([1]).
 struct DevSeg {
-    int L, S, nQp, carry_f, carry_b;
-    const void *G, *H;    // S*K*K forward / backward transfer matrices (compute type)
-    const int *gptr;      // S+1: gamma COO entries of segment s are [gptr[s], gptr[s+1])
+    int L, S, LP, carry_f, carry_b;
+    const void *Lr[2], *Ur[2], *dinv[2];
+    const void *G[2], *H[2];  // S*K*K forward / backward segment transfer matrices
+    const int *gptr;          // S+1: gamma COO entries of segment s are [gptr[s], gptr[s+1])
 };
 
 // Packed constants uploaded once at create ("copy the result
-// to the device").  Floating-point sections exist in fp64 ([0]) and fp32 ([1]).
+// to the device").
 struct DevPlan {
-    int n, nQ, s_lo, k, K;         // order, Q order, Q offset, delta order, kernel band
-    int nQpa;                      // stride of the padded factor arrays
-    int lam_nnz, gam_nnz;          // Lambda CSR / gamma COO sizes
-    const void *Lr[2];             // K arrays of nQpa: L(i, i-1-m) at [m*nQpa + i]
-    const void *Ur[2];             // K arrays of nQpa: U'(i, i+1+m) at [m*nQpa + i]
-    const void *dinv[2];           // nQpa (1 on padding rows)
+    int n, nQ, s_lo, k, K;   // order, Q order, Q offset, delta order, kernel band
+    int lam_nnz, gam_nnz;    // Lambda CSR / gamma COO sizes
     const void *lam_v[2], *gam_v[2], *dlu[2], *dscale[2];
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
-    DevSeg seg[2];                 // [0] fp64 kernels, [1] fp32 kernels
+    DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),
+                             // [2] warp-per-RHS kernel (odd L; S == 0 if unavailable)
 };
 
 struct SolveArgs {

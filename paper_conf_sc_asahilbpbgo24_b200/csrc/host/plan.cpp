@@ -553,8 +553,16 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
     for (auto &c : cands) {
         SplitResult r = try_split(P, c.first, c.second);
         if (r.code) { why = r.msg; why_code = r.code; continue; }
-        build_segplan(P, P.seg[0], 32);
-        build_segplan(P, P.seg[1], 64);
+        build_segplan(P, P.seg[0], 36);
+        build_segplan(P, P.seg[1], 72);
+        {   // warp-per-RHS kernel: odd L (conflict-free smem transpose), S <= 32
+            const int need = std::max(P.K, (P.nQ + 31) / 32);
+            int Lpc = 0;
+            for (int cand : {3, 5, 9, 17, 33, 63})  // instantiated in solve_kernels.cu
+                if (cand >= need) { Lpc = cand; break; }
+            if (Lpc) build_segplan(P, P.seg[2], Lpc);
+            else P.seg[2] = SegPlan();
+        }
         // self-check: residual of the equilibrated system with 4 random RHS
         const int nb = 4;
         std::vector<double> b((size_t)n * nb), x;

@@ -61,8 +61,10 @@ struct Plan {
     std::vector<double> dprime;     // k*k delta' = delta - lambda beta
     std::vector<double> dlu;        // k*k LU of delta' (getrf, partial pivoting)
     std::vector<int> dpiv;          // k
-    // ---- segment plans: [0] fp64 kernels (L=32), [1] fp32 kernels (L=64)
-    SegPlan seg[2];
+    // ---- segment plans: [0] batch-contiguous fp64 kernel (L=36), [1] batch-
+    //      contiguous fp32 kernel (L=72), [2] point-contiguous warp-per-RHS
+    //      kernel (32 lanes = segments, odd L; S = 0 if nQ is too large)
+    SegPlan seg[3];
 };
 
 struct Status {

@@ -102,18 +102,21 @@ def test_parity_point_contiguous(torch_cuda, n_points, dtype):
     assert rel_coef_error(got, ref) <= (TOL64 if dtype == np.float64 else TOL32)
 
 
-def test_strided_equals_contiguous_bitwise(torch_cuda):
-    """The same RHS in batch-contiguous and point-contiguous layouts give the
-    same bits (same per-RHS arithmetic)."""
+def test_strided_matches_contiguous(torch_cuda):
+    """The same RHS in batch-contiguous (tile kernel) and point-contiguous
+    (warp kernel) layouts agree to rounding.  The two kernels use different
+    segment lengths, so the bits may differ."""
     torch = torch_cuda
-    sb, _ = make(3, 1024, PERIODIC, "uniform")
+    sb, o = make(3, 1024, PERIODIC, "uniform")
     b = inputs.rhs(sb.n, 96, seed=5)
     t1 = torch.from_numpy(b).cuda()
     t2 = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()
     sb.solve_(t1)
     sb.solve_(t2)
     torch.cuda.synchronize()
-    assert torch.equal(t1, t2.t())
+    x1, x2 = t1.cpu().numpy(), t2.cpu().numpy().T
+    assert rel_coef_error(x1, x2) <= 1e-14
+    assert rel_coef_error(x2, o.solve(b)) <= TOL64
 
 
 def test_general_strided_subslice(torch_cuda):
