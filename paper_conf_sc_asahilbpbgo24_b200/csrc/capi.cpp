@@ -120,6 +120,16 @@ int upload(spline_builder *h) {
     sb::DevPlan &d = h->dp;
     d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K;
     d.lam_nnz = (int)P.Lam_v.size(); d.gam_nnz = (int)P.gam_v.size();
+    {   // rows the corner step reads: delta rows (b1) and Lambda columns (b0)
+        int head = 0, tail = 0;
+        auto note = [&](int row) {
+            if (row < P.n / 2) head = std::max(head, row + 1);
+            else tail = std::max(tail, P.n - row);
+        };
+        for (int r : P.drow) note(r);
+        for (int c : P.Lam_c) note(P.s_lo + c);
+        d.corner_rows = k > 0 ? std::max(head, tail) : 0;
+    }
     for (int c = 0; c < 2; ++c) {
         d.lam_v[c] = at(oLam[c]); d.gam_v[c] = at(oGam[c]); d.dlu[c] = at(oDlu[c]); d.dscale[c] = at(oDs[c]);
     }

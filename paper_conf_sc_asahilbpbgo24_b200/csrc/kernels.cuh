@@ -52,10 +52,13 @@ struct KParams {
     void *rhs;
     int64_t batch, bstride, pstride;
     int ntiles, nbox, boxr, ncw;     // tiles, TMA boxes per tile, rows per box, compute warps
-    int empty_count[NBOXMAX];        // arrivals that free box c (reader warps + corner warp)
+    int empty_count[NBOXMAX];        // arrivals that free box c (reader warps; corner warp if none)
+    int corner_arrive_mask;          // boxes without a compute-warp reader: the corner warp frees them
+    int cbox;                        // rows of each corner box (0: corner reads the main tile)
     // dynamic shared memory offsets (bytes)
     int off_buf, off_L, off_U, off_dinv, off_G, off_H, off_fend, off_bbeg, off_x1, off_lamptr, off_lamc, off_lamv,
-        off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, smem_total;
+        off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, off_cbuf,
+        smem_total;
     int wbuf_pitch;                  // warp kernel: elements per per-warp row buffer
 };
 
@@ -108,87 +111,89 @@ template <> struct Vec2<double> { using type = double2; };
 template <> struct Vec2<float> { using type = float2; };
 
 // ------------------------------------------------- per-thread segment math
-// Factor access: f[m*ms + i] for band index m (0..K-1) and local row i.
+// Each thread runs NV independent chains (NV right-hand sides) over the same
+// L rows; v[i][q] is row i of RHS q.  Factor access: f[m*ms + i] for band
+// index m (0..K-1) and local row i; one factor load serves all NV chains.
 // PAIRS: rows (i, i+1) are read with one 2-wide load (pitch even, i even).
+// Inside each row the newest state enters the FMA chain last (1-FMA critical
+// path per row).
+
+template <typename C, int K, bool PAIRS>
+__device__ __forceinline__ void load_band(const C *f, int ms, int i, C (&f0)[K], C (&f1)[K]) {
+#pragma unroll
+    for (int m = 0; m < K; ++m) {
+        if constexpr (PAIRS) {
+            const auto w = *reinterpret_cast<const typename Vec2<C>::type *>(f + m * ms + i);
+            f0[m] = w.x;
+            f1[m] = w.y;
+        } else {
+            f0[m] = f[m * ms + i];
+            f1[m] = C(0);
+        }
+    }
+}
 
 // local forward sweep, zero inflow: y_i = b_i - sum_m L(i,i-1-m) y_{i-1-m}
-template <typename C, int K, int L, bool PAIRS>
-__device__ __forceinline__ void fwd_local(C (&v)[L], const C *fL, int ms, C (&st)[K]) {
+template <typename C, int K, int L, int NV, bool PAIRS>
+__device__ __forceinline__ void fwd_local(C (&v)[L][NV], const C *fL, int ms, C (&st)[K][NV]) {
 #pragma unroll
-    for (int m = 0; m < K; ++m) st[m] = C(0);
+    for (int m = 0; m < K; ++m)
+#pragma unroll
+        for (int q = 0; q < NV; ++q) st[m][q] = C(0);
 #pragma unroll
     for (int i = 0; i < L; i += (PAIRS ? 2 : 1)) {
         C l0[K], l1[K];
+        load_band<C, K, PAIRS>(fL, ms, i, l0, l1);
 #pragma unroll
-        for (int m = 0; m < K; ++m) {
-            if constexpr (PAIRS) {
-                const auto w = *reinterpret_cast<const typename Vec2<C>::type *>(fL + m * ms + i);
-                l0[m] = w.x;
-                l1[m] = w.y;
-            } else {
-                l0[m] = fL[m * ms + i];
+        for (int h = 0; h < (PAIRS ? 2 : 1); ++h) {
+#pragma unroll
+            for (int q = 0; q < NV; ++q) {
+                C acc = v[i + h][q];
+#pragma unroll
+                for (int m = K - 1; m >= 0; --m) acc = fma(-(h ? l1[m] : l0[m]), st[m][q], acc);
+#pragma unroll
+                for (int m = K - 1; m > 0; --m) st[m][q] = st[m - 1][q];
+                st[0][q] = acc;
+                v[i + h][q] = acc;
             }
-        }
-#pragma unroll
-        for (int q = 0; q < (PAIRS ? 2 : 1); ++q) {
-            C acc = v[i + q];
-#pragma unroll
-            for (int m = 0; m < K; ++m) acc = fma(-(q ? l1[m] : l0[m]), st[m], acc);
-#pragma unroll
-            for (int m = K - 1; m > 0; --m) st[m] = st[m - 1];
-            st[0] = acc;
-            v[i + q] = acc;
         }
     }
 }
 
 // forward correction chain c_i = -sum_m L(i,i-1-m) c_{i-1-m}, c(a-1-m) = cin[m];  y_i += c_i
-template <typename C, int K, int L, bool PAIRS>
-__device__ __forceinline__ void fwd_correct(C (&v)[L], const C *fL, int ms, C (&cin)[K]) {
+template <typename C, int K, int L, int NV, bool PAIRS>
+__device__ __forceinline__ void fwd_correct(C (&v)[L][NV], const C *fL, int ms, C (&cin)[K][NV]) {
 #pragma unroll
     for (int i = 0; i < L; i += (PAIRS ? 2 : 1)) {
         C l0[K], l1[K];
+        load_band<C, K, PAIRS>(fL, ms, i, l0, l1);
 #pragma unroll
-        for (int m = 0; m < K; ++m) {
-            if constexpr (PAIRS) {
-                const auto w = *reinterpret_cast<const typename Vec2<C>::type *>(fL + m * ms + i);
-                l0[m] = w.x;
-                l1[m] = w.y;
-            } else {
-                l0[m] = fL[m * ms + i];
+        for (int h = 0; h < (PAIRS ? 2 : 1); ++h) {
+#pragma unroll
+            for (int q = 0; q < NV; ++q) {
+                C c = C(0);
+#pragma unroll
+                for (int m = K - 1; m >= 0; --m) c = fma(-(h ? l1[m] : l0[m]), cin[m][q], c);
+#pragma unroll
+                for (int m = K - 1; m > 0; --m) cin[m][q] = cin[m - 1][q];
+                cin[0][q] = c;
+                v[i + h][q] += c;
             }
-        }
-#pragma unroll
-        for (int q = 0; q < (PAIRS ? 2 : 1); ++q) {
-            C c = C(0);
-#pragma unroll
-            for (int m = 0; m < K; ++m) c = fma(-(q ? l1[m] : l0[m]), cin[m], c);
-#pragma unroll
-            for (int m = K - 1; m > 0; --m) cin[m] = cin[m - 1];
-            cin[0] = c;
-            v[i + q] += c;
         }
     }
 }
 
 // local backward sweep, zero outflow: x_i = y_i dinv_i - sum_m U'(i,i+1+m) x_{i+1+m}
-template <typename C, int K, int L, bool PAIRS>
-__device__ __forceinline__ void bwd_local(C (&v)[L], const C *fU, const C *fD, int ms, C (&st)[K]) {
+template <typename C, int K, int L, int NV, bool PAIRS>
+__device__ __forceinline__ void bwd_local(C (&v)[L][NV], const C *fU, const C *fD, int ms, C (&st)[K][NV]) {
 #pragma unroll
-    for (int m = 0; m < K; ++m) st[m] = C(0);
+    for (int m = 0; m < K; ++m)
+#pragma unroll
+        for (int q = 0; q < NV; ++q) st[m][q] = C(0);
 #pragma unroll
     for (int i = L - (PAIRS ? 2 : 1); i >= 0; i -= (PAIRS ? 2 : 1)) {
         C u0[K], u1[K], d0, d1 = C(0);
-#pragma unroll
-        for (int m = 0; m < K; ++m) {
-            if constexpr (PAIRS) {
-                const auto w = *reinterpret_cast<const typename Vec2<C>::type *>(fU + m * ms + i);
-                u0[m] = w.x;
-                u1[m] = w.y;
-            } else {
-                u0[m] = fU[m * ms + i];
-            }
-        }
+        load_band<C, K, PAIRS>(fU, ms, i, u0, u1);
         if constexpr (PAIRS) {
             const auto w = *reinterpret_cast<const typename Vec2<C>::type *>(fD + i);
             d0 = w.x;
@@ -197,43 +202,40 @@ __device__ __forceinline__ void bwd_local(C (&v)[L], const C *fU, const C *fD, i
             d0 = fD[i];
         }
 #pragma unroll
-        for (int q = (PAIRS ? 1 : 0); q >= 0; --q) {
-            C acc = v[i + q] * (q ? d1 : d0);
+        for (int h = (PAIRS ? 1 : 0); h >= 0; --h) {
 #pragma unroll
-            for (int m = 0; m < K; ++m) acc = fma(-(q ? u1[m] : u0[m]), st[m], acc);
+            for (int q = 0; q < NV; ++q) {
+                C acc = v[i + h][q] * (h ? d1 : d0);
 #pragma unroll
-            for (int m = K - 1; m > 0; --m) st[m] = st[m - 1];
-            st[0] = acc;
-            v[i + q] = acc;
+                for (int m = K - 1; m >= 0; --m) acc = fma(-(h ? u1[m] : u0[m]), st[m][q], acc);
+#pragma unroll
+                for (int m = K - 1; m > 0; --m) st[m][q] = st[m - 1][q];
+                st[0][q] = acc;
+                v[i + h][q] = acc;
+            }
         }
     }
 }
 
 // backward correction chain c_i = -sum_m U'(i,i+1+m) c_{i+1+m}, c(a+L+m) = co[m];  x_i += c_i
-template <typename C, int K, int L, bool PAIRS>
-__device__ __forceinline__ void bwd_correct(C (&v)[L], const C *fU, int ms, C (&co)[K]) {
+template <typename C, int K, int L, int NV, bool PAIRS>
+__device__ __forceinline__ void bwd_correct(C (&v)[L][NV], const C *fU, int ms, C (&co)[K][NV]) {
 #pragma unroll
     for (int i = L - (PAIRS ? 2 : 1); i >= 0; i -= (PAIRS ? 2 : 1)) {
         C u0[K], u1[K];
+        load_band<C, K, PAIRS>(fU, ms, i, u0, u1);
 #pragma unroll
-        for (int m = 0; m < K; ++m) {
-            if constexpr (PAIRS) {
-                const auto w = *reinterpret_cast<const typename Vec2<C>::type *>(fU + m * ms + i);
-                u0[m] = w.x;
-                u1[m] = w.y;
-            } else {
-                u0[m] = fU[m * ms + i];
+        for (int h = (PAIRS ? 1 : 0); h >= 0; --h) {
+#pragma unroll
+            for (int q = 0; q < NV; ++q) {
+                C c = C(0);
+#pragma unroll
+                for (int m = K - 1; m >= 0; --m) c = fma(-(h ? u1[m] : u0[m]), co[m][q], c);
+#pragma unroll
+                for (int m = K - 1; m > 0; --m) co[m][q] = co[m - 1][q];
+                co[0][q] = c;
+                v[i + h][q] += c;
             }
-        }
-#pragma unroll
-        for (int q = (PAIRS ? 1 : 0); q >= 0; --q) {
-            C c = C(0);
-#pragma unroll
-            for (int m = 0; m < K; ++m) c = fma(-(q ? u1[m] : u0[m]), co[m], c);
-#pragma unroll
-            for (int m = K - 1; m > 0; --m) co[m] = co[m - 1];
-            co[0] = c;
-            v[i + q] += c;
         }
     }
 }
@@ -285,12 +287,26 @@ __device__ __forceinline__ void stage_constants(const KParams &p, const DevSeg &
 }
 
 // ========================================================= tile kernel
-template <typename T, int K, int L, int R, int LOADER>
+// NV right-hand sides of one row as one vector access
+template <typename T, int NV> struct VecN { using type = T; };
+template <> struct VecN<double, 2> { using type = double2; };
+template <> struct VecN<float, 2> { using type = float2; };
+template <> struct VecN<float, 4> { using type = float4; };
+
+// right-hand sides per compute thread of the tile kernel (1: one chain per
+// thread; 2/4 were measured slower -- per-segment overheads and carry smem grow)
+constexpr int tile_nv(int /*esz*/) { return 1; }
+
+template <typename T, int K, int L, int R, int NV, int LOADER>
 __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
-    sb_tile_kernel(const __grid_constant__ KParams p, const __grid_constant__ CUtensorMap tmap) {
+    sb_tile_kernel(const __grid_constant__ KParams p, const __grid_constant__ CUtensorMap tmap,
+                   const __grid_constant__ CUtensorMap tmap_c) {
     using C = T;  // compute in the storage precision
     constexpr int CI = sizeof(T) == 8 ? 0 : 1;
-    constexpr int SPW = 32 / R;  // segments per compute warp
+    constexpr int CPR = 32 / R;   // corner lanes per RHS
+    constexpr int RP = R / NV;    // RHS groups per tile (a thread owns NV adjacent RHS)
+    constexpr int SPW = 32 / RP;  // segments per compute warp
+    static_assert(NV * (int)sizeof(T) <= 16, "NV RHS form one vector of at most 16 B");
     extern __shared__ __align__(1024) unsigned char smem[];
     const DevPlan &P = p.P;
     const DevSeg &G = P.seg[CI];
@@ -322,7 +338,11 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + p.off_mbar);
     uint64_t *empty = full + NBOXMAX;
     uint64_t *x1full = empty + NBOXMAX;
+    uint64_t *cfull = x1full + 2;  // corner boxes, double-buffered
     T *buf = reinterpret_cast<T *>(smem + p.off_buf);
+    T *cbuf = reinterpret_cast<T *>(smem + p.off_cbuf);  // [2][2 boxes][cbox rows][R]
+    const int cbox = p.cbox;
+    const bool use_cbox = LOADER == LOAD_TMA && cbox > 0;
     T *gout = reinterpret_cast<T *>(p.rhs);
     const int64_t ps = p.pstride;
     const uint32_t box_bytes = (uint32_t)(boxr * R * sizeof(T));
@@ -334,33 +354,55 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         }
         mbar_init(x1full + 0, 1);
         mbar_init(x1full + 1, 1);
+        mbar_init(cfull + 0, 1);
+        mbar_init(cfull + 1, 1);
         fence_mbar_init();
         if (LOADER == LOAD_TMA) prefetch_tmap(&tmap);
+        if (use_cbox) prefetch_tmap(&tmap_c);
     }
     stage_constants<C, K>(p, G, smem, tid, blockDim.x);
     __syncthreads();
 
     if (warp == ncw) {
         // ===================== corner + producer warp (runs one tile ahead)
+        // The corner of tile t+1 needs only its head/tail rows: they arrive in two
+        // small "corner boxes" issued one tile early, so x1(t+1) is ready before
+        // the compute warps reach tile t+1 (the main load re-reads those rows from L2).
         const int part = lane / R, rr = lane % R;
+        const uint32_t cbytes = (uint32_t)(2 * cbox * R * sizeof(T));
+        auto issue_cbox = [&](int t, int b) {
+            T *dst = cbuf + (size_t)b * 2 * cbox * R;
+            mbar_arrive_expect_tx(cfull + b, cbytes);
+            tma_load_2d(dst, &tmap_c, cfull + b, t * R, 0);
+            tma_load_2d(dst + (size_t)cbox * R, &tmap_c, cfull + b, t * R, P.n - cbox);
+        };
+        if (use_cbox && lane == 0 && (int)blockIdx.x < p.ntiles) issue_cbox(blockIdx.x, 0);
         int it = 0;
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
             if (LOADER == LOAD_TMA) {
-                if (lane == 0)
+                if (lane == 0) {
                     for (int c = 0; c < nbox; ++c) {
                         if (it > 0) mbar_wait(empty + c, (it - 1) & 1);
                         mbar_arrive_expect_tx(full + c, box_bytes);
                         tma_load_2d(buf + (size_t)c * boxr * R, &tmap, full + c, tile * R, c * boxr);
                     }
-                for (int c = 0; c < nbox; ++c) mbar_wait(full + c, it & 1);
+                    if (use_cbox && tile + (int)gridDim.x < p.ntiles) issue_cbox(tile + gridDim.x, (it + 1) & 1);
+                }
+                if (use_cbox) mbar_wait(cfull + (it & 1), (it >> 1) & 1);
+                else
+                    for (int c = 0; c < nbox; ++c) mbar_wait(full + c, it & 1);
             } else if (it > 0) {
                 mbar_wait(empty + 0, (it - 1) & 1);  // all compute warps finished tile it-1
             }
+            const T *cb = cbuf + (size_t)(it & 1) * 2 * cbox * R;
             const int64_t ccol = (int64_t)tile * R + rr;
             const bool clive = ccol < p.batch;
             const T *ccolp = gout + ccol * p.bstride;
             auto ldb = [&](int row) -> C {
-                if (LOADER == LOAD_TMA) return (C)buf[(size_t)row * R + rr];
+                if (LOADER == LOAD_TMA) {
+                    if (use_cbox) return (C)cb[(size_t)(row < cbox ? row : cbox + row - (P.n - cbox)) * R + rr];
+                    return (C)buf[(size_t)row * R + rr];
+                }
                 return clive ? (C)ccolp[(int64_t)row * ps] : C(0);
             };
             C *x1 = sx1 + (it & 1) * R * k + rr * k;
@@ -370,13 +412,13 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 const int e1 = slamptr[d + 1];
                 // 4 independent partial sums keep the dependent smem loads in flight
                 C a1 = C(0), a2 = C(0), a3 = C(0);
-                for (; e + 3 * SPW < e1; e += 4 * SPW) {
+                for (; e + 3 * CPR < e1; e += 4 * CPR) {
                     acc = fma(-slamv[e], ldb(s_lo + slamc[e]), acc);
-                    a1 = fma(-slamv[e + SPW], ldb(s_lo + slamc[e + SPW]), a1);
-                    a2 = fma(-slamv[e + 2 * SPW], ldb(s_lo + slamc[e + 2 * SPW]), a2);
-                    a3 = fma(-slamv[e + 3 * SPW], ldb(s_lo + slamc[e + 3 * SPW]), a3);
+                    a1 = fma(-slamv[e + CPR], ldb(s_lo + slamc[e + CPR]), a1);
+                    a2 = fma(-slamv[e + 2 * CPR], ldb(s_lo + slamc[e + 2 * CPR]), a2);
+                    a3 = fma(-slamv[e + 3 * CPR], ldb(s_lo + slamc[e + 3 * CPR]), a3);
                 }
-                for (; e < e1; e += SPW) acc = fma(-slamv[e], ldb(s_lo + slamc[e]), acc);
+                for (; e < e1; e += CPR) acc = fma(-slamv[e], ldb(s_lo + slamc[e]), acc);
                 acc += (a1 + a2) + a3;
 #pragma unroll
                 for (int off = R; off < 32; off *= 2) acc += __shfl_xor_sync(0xffffffffu, acc, off);
@@ -391,15 +433,18 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             if (lane == 0) {
                 mbar_arrive(x1full + (it & 1));
                 if (LOADER == LOAD_TMA)
-                    for (int c = 0; c < nbox; ++c) mbar_arrive(empty + c);
+                    for (int c = 0; c < nbox; ++c)
+                        if (!use_cbox || ((p.corner_arrive_mask >> c) & 1)) mbar_arrive(empty + c);
             }
         }
         return;
     }
 
     // ============================================== compute warps
-    const int r = tid % R;
-    const int s = tid / R;
+    using V = typename VecN<T, NV>::type;
+    const int rp = tid % RP;
+    const int s = tid / RP;
+    const int r0 = rp * NV;  // first of this thread's NV right-hand sides in the tile
     const bool active = s < S;
     const int a = s * L;
     const bool full_seg = a + L <= nQ;
@@ -411,119 +456,161 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     int c_lo = 0, c_hi = -1;
     {
         const int s0 = warp * SPW;
-        const int r0 = s_lo + s0 * L;
-        const int r1 = s_lo + min((s0 + SPW) * L, nQ) - 1;
-        if (s0 < S && r1 >= r0) {
-            c_lo = r0 / boxr;
-            c_hi = r1 / boxr;
+        const int rr0 = s_lo + s0 * L;
+        const int rr1 = s_lo + min((s0 + SPW) * L, nQ) - 1;
+        if (s0 < S && rr1 >= rr0) {
+            c_lo = rr0 / boxr;
+            c_hi = rr1 / boxr;
         }
     }
     const int nthr_c = ncw * 32;
     int it = 0;
     for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
-        const int64_t col = (int64_t)tile * R + r;
-        const bool live = active && col < p.batch;
-        T *gcol = gout + col * p.bstride;
-        C v[L];
+        const int64_t col0 = (int64_t)tile * R + r0;
+        // right-hand sides of this thread that exist (0..NV)
+        const int nlive = active ? (int)max((int64_t)0, min((int64_t)NV, p.batch - col0)) : 0;
+        T *gcol = gout + col0 * p.bstride;
+        C v[L][NV];
         // ---------- own segment of b0 into registers
         if (LOADER == LOAD_TMA) {
             for (int c = c_lo; c <= c_hi; ++c) mbar_wait(full + c, it & 1);
-            const T *src = buf + (size_t)(s_lo + a) * R + r;
+            const T *src = buf + (size_t)(s_lo + a) * R + r0;
             if (full_seg) {
 #pragma unroll
-                for (int i = 0; i < L; ++i) v[i] = (C)src[(size_t)i * R];
+                for (int i = 0; i < L; ++i) {
+                    const V w = *reinterpret_cast<const V *>(src + (size_t)i * R);
+                    const T *pw = reinterpret_cast<const T *>(&w);
+#pragma unroll
+                    for (int q = 0; q < NV; ++q) v[i][q] = (C)pw[q];
+                }
             } else {
 #pragma unroll
-                for (int i = 0; i < L; ++i) v[i] = (active && a + i < nQ) ? (C)src[(size_t)i * R] : C(0);
+                for (int i = 0; i < L; ++i) {
+                    if (active && a + i < nQ) {
+                        const V w = *reinterpret_cast<const V *>(src + (size_t)i * R);
+                        const T *pw = reinterpret_cast<const T *>(&w);
+#pragma unroll
+                        for (int q = 0; q < NV; ++q) v[i][q] = (C)pw[q];
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < NV; ++q) v[i][q] = C(0);
+                    }
+                }
             }
             __syncwarp();
             if (lane == 0)
                 for (int c = c_lo; c <= c_hi; ++c) mbar_arrive(empty + c);
         } else {
             const T *src = gcol + (int64_t)(s_lo + a) * ps;
-            if (full_seg && live) {
 #pragma unroll
-                for (int i = 0; i < L; ++i) v[i] = (C)__ldcs(src + (int64_t)i * ps);
-            } else {
+            for (int i = 0; i < L; ++i)
 #pragma unroll
-                for (int i = 0; i < L; ++i) v[i] = (live && a + i < nQ) ? (C)__ldcs(src + (int64_t)i * ps) : C(0);
-            }
+                for (int q = 0; q < NV; ++q)
+                    v[i][q] = (q < nlive && a + i < nQ) ? (C)__ldcs(src + (int64_t)i * ps + q * p.bstride) : C(0);
         }
         // ---------- b0 -= gamma x1 (only segments holding gamma rows wait for the corner warp)
         if (active && sgptr[s] < sgptr[s + 1]) {
             mbar_wait(x1full + (it & 1), (it >> 1) & 1);
-            const C *x1 = sx1 + (it & 1) * R * k + r * k;
+            const C *x1 = sx1 + (it & 1) * R * k + r0 * k;
             for (int e = sgptr[s]; e < sgptr[s + 1]; ++e) {
                 const int i = sgamr[e] - a;
-                const C dv = sgamv[e] * x1[sgamc[e]];
+                const int dc = sgamc[e];
+                const C gv = sgamv[e];
 #pragma unroll
                 for (int j = 0; j < L; ++j)
-                    if (j == i) v[j] -= dv;
+                    if (j == i)
+#pragma unroll
+                        for (int q = 0; q < NV; ++q) v[j][q] = fma(-gv, x1[q * k + dc], v[j][q]);
             }
         }
         // ---------- local forward sweep, publish end state
-        C st[K];
-        fwd_local<C, K, L, true>(v, fL, ms, st);
+        C st[K][NV];
+        fwd_local<C, K, L, NV, true>(v, fL, ms, st);
         if (active)
 #pragma unroll
-            for (int j = 0; j < K; ++j) sfend[(s * R + r) * K + j] = st[j];
+            for (int q = 0; q < NV; ++q)
+#pragma unroll
+                for (int j = 0; j < K; ++j) sfend[(s * R + r0 + q) * K + j] = st[j][q];
         named_bar(1, nthr_c);  // B2
         // ---------- forward carry (true y at rows a-1..a-K) + correction chain
         if (active && s > 0) {
-            C cin[K];
+            C cin[K][NV];
 #pragma unroll
-            for (int m = 0; m < K; ++m) cin[m] = C(0);
+            for (int m = 0; m < K; ++m)
+#pragma unroll
+                for (int q = 0; q < NV; ++q) cin[m][q] = C(0);
             for (int t = max(0, s - G.carry_f); t < s; ++t) {
-                C nw[K];
+                C nw[K][NV];
 #pragma unroll
-                for (int j = 0; j < K; ++j) {
-                    C acc = sfend[(t * R + r) * K + j];
+                for (int j = 0; j < K; ++j)
 #pragma unroll
-                    for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m], acc);
-                    nw[j] = acc;
-                }
+                    for (int q = 0; q < NV; ++q) {
+                        C acc = sfend[(t * R + r0 + q) * K + j];
 #pragma unroll
-                for (int j = 0; j < K; ++j) cin[j] = nw[j];
+                        for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m][q], acc);
+                        nw[j][q] = acc;
+                    }
+#pragma unroll
+                for (int j = 0; j < K; ++j)
+#pragma unroll
+                    for (int q = 0; q < NV; ++q) cin[j][q] = nw[j][q];
             }
-            fwd_correct<C, K, L, true>(v, fL, ms, cin);
+            fwd_correct<C, K, L, NV, true>(v, fL, ms, cin);
         }
         // ---------- local backward sweep, publish begin state
-        bwd_local<C, K, L, true>(v, fU, fD, ms, st);
+        bwd_local<C, K, L, NV, true>(v, fU, fD, ms, st);
         if (active)
 #pragma unroll
-            for (int j = 0; j < K; ++j) sbbeg[(s * R + r) * K + j] = st[j];
+            for (int q = 0; q < NV; ++q)
+#pragma unroll
+                for (int j = 0; j < K; ++j) sbbeg[(s * R + r0 + q) * K + j] = st[j][q];
         named_bar(1, nthr_c);  // B3
         // ---------- backward carry (true x at rows a+L..a+L+K-1) + correction chain
         if (active && s < S - 1) {
-            C co[K];
+            C co[K][NV];
 #pragma unroll
-            for (int m = 0; m < K; ++m) co[m] = C(0);
+            for (int m = 0; m < K; ++m)
+#pragma unroll
+                for (int q = 0; q < NV; ++q) co[m][q] = C(0);
             for (int t = min(S - 1, s + G.carry_b); t > s; --t) {
-                C nw[K];
+                C nw[K][NV];
 #pragma unroll
-                for (int j = 0; j < K; ++j) {
-                    C acc = sbbeg[(t * R + r) * K + j];
+                for (int j = 0; j < K; ++j)
 #pragma unroll
-                    for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m], acc);
-                    nw[j] = acc;
-                }
+                    for (int q = 0; q < NV; ++q) {
+                        C acc = sbbeg[(t * R + r0 + q) * K + j];
 #pragma unroll
-                for (int j = 0; j < K; ++j) co[j] = nw[j];
+                        for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m][q], acc);
+                        nw[j][q] = acc;
+                    }
+#pragma unroll
+                for (int j = 0; j < K; ++j)
+#pragma unroll
+                    for (int q = 0; q < NV; ++q) co[j][q] = nw[j][q];
             }
-            bwd_correct<C, K, L, true>(v, fU, ms, co);
+            bwd_correct<C, K, L, NV, true>(v, fU, ms, co);
         }
-        // ---------- store x0 straight from registers.  DIRECT mode: the corner warp
-        // reads b0 from HBM, so no row of this tile is overwritten before x1 is done.
+        // ---------- store x0 straight from registers (one 16-B vector per row).
+        // DIRECT mode: the corner warp reads b0 from HBM, so no row of this tile is
+        // overwritten before x1 is done.
         if (LOADER == LOAD_DIRECT && k > 0) mbar_wait(x1full + (it & 1), (it >> 1) & 1);
-        if (live) {
+        if (nlive > 0) {
             T *dst = gcol + (int64_t)(s_lo + a) * ps;
-            if (full_seg) {
+            if (LOADER == LOAD_TMA && nlive == NV && full_seg) {
 #pragma unroll
-                for (int i = 0; i < L; ++i) __stcs(dst + (int64_t)i * ps, (T)v[i]);
+                for (int i = 0; i < L; ++i) {
+                    V w;
+                    T *pw = reinterpret_cast<T *>(&w);
+#pragma unroll
+                    for (int q = 0; q < NV; ++q) pw[q] = (T)v[i][q];
+                    __stcs(reinterpret_cast<V *>(dst + (int64_t)i * ps), w);
+                }
             } else {
 #pragma unroll
                 for (int i = 0; i < L; ++i)
-                    if (a + i < nQ) __stcs(dst + (int64_t)i * ps, (T)v[i]);
+#pragma unroll
+                    for (int q = 0; q < NV; ++q)
+                        if (q < nlive && a + i < nQ) __stcs(dst + (int64_t)i * ps + q * p.bstride, (T)v[i][q]);
             }
         }
         if (LOADER == LOAD_DIRECT) {  // tile done: lets the corner warp move to tile it+1
@@ -616,58 +703,58 @@ __global__ void __launch_bounds__(256)
             __syncwarp();
         }
         // ---------- own segment into registers (odd L: conflict-free)
-        C v[L];
+        C v[L][1];
 #pragma unroll
-        for (int i = 0; i < L; ++i) v[i] = (active && a + i < nQ) ? rowbuf[s_lo + a + i] : C(0);
+        for (int i = 0; i < L; ++i) v[i][0] = (active && a + i < nQ) ? rowbuf[s_lo + a + i] : C(0);
         // ---------- forward: local sweep, carry by shuffles, correction chain
-        C st[K];
-        fwd_local<C, K, L, false>(v, fL, ms, st);
+        C st[K][1];
+        fwd_local<C, K, L, 1, false>(v, fL, ms, st);
         {
-            C cin[K];
+            C cin[K][1];
 #pragma unroll
-            for (int m = 0; m < K; ++m) cin[m] = C(0);
+            for (int m = 0; m < K; ++m) cin[m][0] = C(0);
             for (int w = G.carry_f; w >= 1; --w) {  // from segment s-w up to s-1
                 const int t = s - w;
                 C nw[K];
 #pragma unroll
                 for (int j = 0; j < K; ++j) {
-                    C acc = __shfl_up_sync(0xffffffffu, st[j], w);
+                    C acc = __shfl_up_sync(0xffffffffu, st[j][0], w);
                     if (t >= 0)
 #pragma unroll
-                        for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m], acc);
+                        for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m][0], acc);
                     nw[j] = t >= 0 ? acc : C(0);
                 }
 #pragma unroll
-                for (int j = 0; j < K; ++j) cin[j] = nw[j];
+                for (int j = 0; j < K; ++j) cin[j][0] = nw[j];
             }
-            if (active && s > 0) fwd_correct<C, K, L, false>(v, fL, ms, cin);
+            if (active && s > 0) fwd_correct<C, K, L, 1, false>(v, fL, ms, cin);
         }
         // ---------- backward: local sweep, carry by shuffles, correction chain
-        bwd_local<C, K, L, false>(v, fU, fD, ms, st);
+        bwd_local<C, K, L, 1, false>(v, fU, fD, ms, st);
         {
-            C co[K];
+            C co[K][1];
 #pragma unroll
-            for (int m = 0; m < K; ++m) co[m] = C(0);
+            for (int m = 0; m < K; ++m) co[m][0] = C(0);
             for (int w = G.carry_b; w >= 1; --w) {  // from segment s+w down to s+1
                 const int t = s + w;
                 C nw[K];
 #pragma unroll
                 for (int j = 0; j < K; ++j) {
-                    C acc = __shfl_down_sync(0xffffffffu, st[j], w);
+                    C acc = __shfl_down_sync(0xffffffffu, st[j][0], w);
                     if (t < S)
 #pragma unroll
-                        for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m], acc);
+                        for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m][0], acc);
                     nw[j] = t < S ? acc : C(0);
                 }
 #pragma unroll
-                for (int j = 0; j < K; ++j) co[j] = nw[j];
+                for (int j = 0; j < K; ++j) co[j][0] = nw[j];
             }
-            if (active && s < S - 1) bwd_correct<C, K, L, false>(v, fU, ms, co);
+            if (active && s < S - 1) bwd_correct<C, K, L, 1, false>(v, fU, ms, co);
         }
         // ---------- back to the row buffer, coalesced store
 #pragma unroll
         for (int i = 0; i < L; ++i)
-            if (active && a + i < nQ) rowbuf[s_lo + a + i] = v[i];
+            if (active && a + i < nQ) rowbuf[s_lo + a + i] = v[i][0];
         __syncwarp();
         if (vec) {
             using V = typename std::conditional<sizeof(T) == 8, double2, float4>::type;
@@ -690,9 +777,9 @@ __global__ void __launch_bounds__(256)
 
 namespace sb {
 // per-TU launchers (tile_f64.cu, tile_f32.cu, warp_f64.cu, warp_f32.cu)
-int launch_tile_f64(int R, int loader, int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads,
+int launch_tile_f64(int R, int loader, int K, const KParams &kp, const CUtensorMap *tm, int grid, int threads,
                     cudaStream_t st, char *err, int errlen);
-int launch_tile_f32(int R, int loader, int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads,
+int launch_tile_f32(int R, int loader, int K, const KParams &kp, const CUtensorMap *tm, int grid, int threads,
                     cudaStream_t st, char *err, int errlen);
 int launch_warp_f64(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 int launch_warp_f32(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
@@ -707,17 +794,17 @@ inline int check_launch(const char *what, char *err, int errlen) {
 }
 
 template <typename T, int K, int L, int R, int LOADER>
-int launch_tile(const KParams &kp, const CUtensorMap &tm, int grid, int threads, cudaStream_t st, char *err,
+int launch_tile(const KParams &kp, const CUtensorMap *tm, int grid, int threads, cudaStream_t st, char *err,
                 int errlen) {
-    auto fn = sb_tile_kernel<T, K, L, R, LOADER>;
+    auto fn = sb_tile_kernel<T, K, L, R, tile_nv(sizeof(T)), LOADER>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total) != cudaSuccess)
         return check_launch("cudaFuncSetAttribute(tile)", err, errlen);
-    fn<<<grid, threads, kp.smem_total, st>>>(kp, tm);
+    fn<<<grid, threads, kp.smem_total, st>>>(kp, tm[0], tm[1]);
     return check_launch("tile kernel launch", err, errlen);
 }
 
 template <typename T, int L, int R, int LOADER>
-int tile_K(int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads, cudaStream_t st, char *err,
+int tile_K(int K, const KParams &kp, const CUtensorMap *tm, int grid, int threads, cudaStream_t st, char *err,
            int errlen) {
     switch (K) {
         case 1: return launch_tile<T, 1, L, R, LOADER>(kp, tm, grid, threads, st, err, errlen);

@@ -1,5 +1,7 @@
 // solve_kernels.cu -- host-side dispatch of the fused kernels (kernels.cuh):
 // layout / tile-width / loader choice, shared-memory layout, TMA descriptor.
+#include <cstdlib>
+
 #include "kernels.cuh"
 
 namespace sb {
@@ -23,7 +25,7 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
-int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes) {
+int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0) {
     size_t o = 0;
     auto take = [&](size_t bytes, size_t al) {
         o = align_up(o, al);
@@ -52,7 +54,8 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_dpiv = take((size_t)k * 4, 16);
     kp.off_dscale = take((size_t)k * esz, 16);
     kp.off_drow = take((size_t)k * 4, 16);
-    kp.off_mbar = take((2 * NBOXMAX + 2) * 8, 8);
+    kp.off_cbuf = take((size_t)4 * cbox * R * esz, 128);
+    kp.off_mbar = take((2 * NBOXMAX + 4) * 8, 8);
     kp.smem_total = (int)align_up(o, 16);
     return kp.smem_total;
 }
@@ -114,7 +117,7 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
     int R = 0, loader = LOAD_DIRECT;
     for (int ci = 0; ci < 2 && !R; ++ci) {
         const int cand = cands[ci];
-        const int ncw = (cand * G.S + 31) / 32;
+        const int ncw = (cand / tile_nv((int)esz) * G.S + 31) / 32;  // RP = R / NV threads per segment
         if ((ncw + 1) * 32 > TILE_MAX_THREADS) continue;
         KParams t = kp;
         if (aligned && a.batch >= cand && nbox <= NBOXMAX && get_encode() &&
@@ -127,38 +130,73 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
         }
     }
     if (!R) return launch_warp(P, a, num_sms, max_smem, err, errlen);  // too large for the tile kernel
-    kp.ncw = (R * G.S + 31) / 32;
+    const int RP = R / tile_nv((int)esz);  // a compute thread owns NV right-hand sides
+    kp.ncw = (RP * G.S + 31) / 32;
     layout_smem(kp, P, G, R, esz, loader == LOAD_TMA ? (size_t)nbox * boxr * R * esz : 0);
     kp.ntiles = (int)((a.batch + R - 1) / R);
     kp.nbox = nbox;
     kp.boxr = boxr;
-    // arrivals that free box c: compute warps whose real rows touch it, plus the corner warp.
-    // DIRECT: empty[0] counts the compute warps that finished a tile.
-    const int spw = 32 / R;
-    for (int c = 0; c < NBOXMAX; ++c) kp.empty_count[c] = loader == LOAD_TMA ? 1 : (c == 0 ? kp.ncw : 1);
-    if (loader == LOAD_TMA)
-    for (int w = 0; w < kp.ncw; ++w) {
-        const int s0 = w * spw;
-        if (s0 >= G.S) continue;
-        const int r0 = P.s_lo + s0 * L;
-        const int r1 = P.s_lo + std::min((s0 + spw) * L, P.nQ) - 1;
-        if (r1 < r0) continue;
-        for (int c = r0 / boxr; c <= r1 / boxr; ++c) kp.empty_count[c]++;
+    // corner boxes: the corner reads only rows [0,cbox) and [n-cbox,n); they are
+    // fetched one tile early with their own (smaller) tensor map
+    int cbox = 0;
+    static const int cbox_env = [] {  // SB_TILE_CBOX=0 disables corner boxes (A/B experiments)
+        const char *e = getenv("SB_TILE_CBOX");
+        return e ? atoi(e) : 1;
+    }();
+    // worth it only when the corner step is heavy enough to delay the gamma warps
+    // (measured: k=1 / 48 nnz C2 loses 4.6 %, k=6 Hermite C3 gains 16 %)
+    const int corner_work = P.lam_nnz / (32 / R) + P.k * P.k;
+    if (loader == LOAD_TMA && P.corner_rows > 0 && cbox_env && (corner_work > 30 || cbox_env > 1)) {
+        cbox = (P.corner_rows + 7) / 8 * 8;
+        KParams t = kp;
+        if (cbox > 256 || 2 * cbox > P.n ||
+            layout_smem(t, P, G, R, esz, (size_t)nbox * boxr * R * esz, cbox) > max_smem)
+            cbox = 0;
     }
-    CUtensorMap tm;
-    memset(&tm, 0, sizeof(tm));
+    kp.cbox = cbox;
+    layout_smem(kp, P, G, R, esz, loader == LOAD_TMA ? (size_t)nbox * boxr * R * esz : 0, cbox);
+    // arrivals that free box c: compute warps whose real rows touch it (+ the corner
+    // warp when it reads the main tile, or when no compute warp reads box c).
+    // DIRECT: empty[0] counts the compute warps that finished a tile.
+    const int spw = 32 / RP;
+    for (int c = 0; c < NBOXMAX; ++c) kp.empty_count[c] = 0;
+    kp.corner_arrive_mask = 0;
     if (loader == LOAD_TMA) {
-        cuuint64_t dims[2] = {(cuuint64_t)a.batch, (cuuint64_t)P.n};
-        cuuint64_t strides[1] = {(cuuint64_t)(a.pstride * (int64_t)esz)};
-        cuuint32_t box[2] = {(cuuint32_t)R, (cuuint32_t)boxr};
-        cuuint32_t estr[2] = {1, 1};
-        CUresult cr = get_encode()(&tm, a.dtype == 0 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
-                                   2, a.rhs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-        if (cr != CUDA_SUCCESS) {
-            snprintf(err, errlen, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
-            return 3;
+        for (int w = 0; w < kp.ncw; ++w) {
+            const int s0 = w * spw;
+            if (s0 >= G.S) continue;
+            const int r0 = P.s_lo + s0 * L;
+            const int r1 = P.s_lo + std::min((s0 + spw) * L, P.nQ) - 1;
+            if (r1 < r0) continue;
+            for (int c = r0 / boxr; c <= r1 / boxr; ++c) kp.empty_count[c]++;
+        }
+        for (int c = 0; c < nbox; ++c)
+            if (cbox == 0 || kp.empty_count[c] == 0) {
+                kp.empty_count[c]++;
+                kp.corner_arrive_mask |= 1 << c;
+            }
+    } else {
+        kp.empty_count[0] = kp.ncw;
+    }
+    for (int c = 0; c < NBOXMAX; ++c)
+        if (kp.empty_count[c] == 0) kp.empty_count[c] = 1;  // unused boxes: any valid count
+    CUtensorMap tm[2];
+    memset(tm, 0, sizeof(tm));
+    if (loader == LOAD_TMA) {
+        for (int q = 0; q < (cbox ? 2 : 1); ++q) {
+            cuuint64_t dims[2] = {(cuuint64_t)a.batch, (cuuint64_t)P.n};
+            cuuint64_t strides[1] = {(cuuint64_t)(a.pstride * (int64_t)esz)};
+            cuuint32_t box[2] = {(cuuint32_t)R, (cuuint32_t)(q == 0 ? boxr : cbox)};
+            cuuint32_t estr[2] = {1, 1};
+            CUresult cr = get_encode()(&tm[q], a.dtype == 0 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64
+                                                            : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                                       2, a.rhs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                       CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            if (cr != CUDA_SUCCESS) {
+                snprintf(err, errlen, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
+                return 3;
+            }
         }
     }
     const int threads = (kp.ncw + 1) * 32;

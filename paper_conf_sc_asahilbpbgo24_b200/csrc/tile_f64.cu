@@ -2,7 +2,7 @@
 #include "kernels.cuh"
 
 namespace sb {
-int launch_tile_f64(int R, int loader, int K, const KParams &kp, const CUtensorMap &tm, int grid, int threads,
+int launch_tile_f64(int R, int loader, int K, const KParams &kp, const CUtensorMap *tm, int grid, int threads,
                     cudaStream_t st, char *err, int errlen) {
     const bool tma = loader == LOAD_TMA;
     if (R == 16) return tma ? tile_K<double, 36, 16, LOAD_TMA>(K, kp, tm, grid, threads, st, err, errlen)
