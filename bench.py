@@ -35,9 +35,12 @@ sys.path.insert(0, ROOT)
 from paper_conf_sc_asahilbpbgo24_b200 import inputs  # noqa: E402
 
 METRIC = "RHS/s and achieved HBM GB/s (% of peak), cubic n=1000, 1e5 RHS, fp64"
+STRONG = {"C5"}            # total batch fixed, sharded over the ranks
+DEVICE_INPUT_ELEMS = 4e8   # above this, inputs are generated on the device (inputs.rhs_device)
+E2E_MAX_RHS = 1_000_000    # the e2e leg moves at most this many RHS through host memory
 
 WORKLOADS = {
-    # name: (degree, n_points, bc, mesh, batch per GPU, dtype, layout, description)
+    # name: (degree, n_points, bc, mesh, batch per GPU (weak) or total (C5, strong), dtype, layout, description)
     "C1": (3, 16, 0, "uniform", 8, "f64", "batch", "C1 cubic uniform periodic n=16 batch=8 fp64"),
     "C2": (3, 1000, 0, "uniform", 100000, "f64", "batch",
            "C2 cubic uniform periodic n=1000 batch=1e5 fp64 batch-contiguous"),
@@ -47,8 +50,8 @@ WORKLOADS = {
            "C4 GYSELA slice f[64][64][32][x=1024] cubic periodic along x, x contiguous, fp64"),
     "C4F32": (3, 1024, 0, "uniform", 131072, "f32", "point",
               "C4 GYSELA slice f[64][64][32][x=1024] cubic periodic along x, x contiguous, fp32"),
-    "C5": (3, 1000, 0, "uniform", 1000000, "f64", "batch",
-           "C5 cubic uniform periodic n=1000, 1e6 RHS per GPU (8e6 over 8 GPUs) fp64"),
+    "C5": (3, 1000, 0, "uniform", 8000000, "f64", "batch",
+           "C5 cubic uniform periodic n=1000, 8e6 RHS in total sharded over the GPUs (strong scaling) fp64"),
 }
 
 
@@ -226,15 +229,28 @@ def main():
     torch.cuda.set_device(local)
     if ws > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    deg, npts, bc, mesh, B, dt, layout, desc = wl
+    from paper_conf_sc_asahilbpbgo24_b200.shard import shard_bounds, weak_bounds
+    deg, npts, bc, mesh, Bspec, dt, layout, desc = wl
+    strong = args.workload in STRONG
+    first, last = shard_bounds(rank, ws, Bspec) if strong else weak_bounds(rank, Bspec)
+    B = last - first                      # this rank's RHS
+    B_total = Bspec if strong else ws * Bspec
     n = inputs.nbasis(deg, npts, bc)
     knots = inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh)
     sb = SplineBuilder(deg, npts, bc, knots)
     esz = 4 if dt == "f32" else 8
-    # this rank's slice of the global batch (weak scaling)
-    host = make_rhs(deg, n, bc, B, rank * B, layout, dt)
-    pristine = torch.from_numpy(host).cuda()
-    x = pristine.clone()
+    tdt = torch.float32 if dt == "f32" else torch.float64
+    on_device = n * B > DEVICE_INPUT_ELEMS and layout == "batch"
+    if on_device:
+        host = None
+        x = inputs.rhs_device(n, B, seed=1234, first=first, dtype=tdt)
+        pristine = None
+        restore = lambda: inputs.rhs_device(n, B, seed=1234, first=first, dtype=tdt, out=x)  # noqa: E731
+    else:
+        host = make_rhs(deg, n, bc, B, first, layout, dt)
+        pristine = torch.from_numpy(host).cuda()
+        x = pristine.clone()
+        restore = lambda: x.copy_(pristine)  # noqa: E731
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -258,7 +274,7 @@ def main():
         done = 0
         for c in range(nchunks):
             m = min(CHUNK, args.steps - done)
-            x.copy_(pristine)
+            restore()
             flush.fill_(c & 0xFF)
             starts[c].record(stream)
             for _ in range(m):
@@ -266,27 +282,30 @@ def main():
             ends[c].record(stream)
             done += m
         barrier()
-    total_ms = float(sum(s.elapsed_time(e) for s, e in zip(starts, ends)))
+    total_ms = float(sum(s_.elapsed_time(e_) for s_, e_ in zip(starts, ends)))
     t_tensor = torch.tensor([total_ms, total_ms / args.steps], device="cuda", dtype=torch.float64)
     if ws > 1:
         dist.all_reduce(t_tensor, op=dist.ReduceOp.MAX)
     total_ms, kern_avg_ms = float(t_tensor[0]), float(t_tensor[1])
     ms_per_step = total_ms / args.steps
-    value = ws * B / (ms_per_step / 1e3)
+    value = B_total / (ms_per_step / 1e3)
     alg_bytes = 2.0 * n * B * esz
-    achieved = alg_bytes / (kern_avg_ms / 1e3) / 1e9
+    achieved = alg_bytes / (kern_avg_ms / 1e3) / 1e9   # per GPU (the slowest rank's kernel time)
     peak, peak_kind = load_peaks()
 
     # end to end through the C ABI with host buffers (pinned), copies in the timed region
     e2e = None
     if not args.no_e2e:
-        hp = torch.from_numpy(host.copy()).pin_memory()
+        Be = min(B, E2E_MAX_RHS)
+        hsrc = host if host is not None else np.ascontiguousarray(x[:, :Be].cpu().numpy())
         if layout == "batch":
+            hsrc = np.ascontiguousarray(hsrc[:, :Be])
+            hp = torch.from_numpy(hsrc.copy()).pin_memory()
             sb.solve_host_(hp)  # warm-up (allocates staging)
             barrier()
             ts = []
             for _ in range(args.e2e_steps):
-                hp.copy_(torch.from_numpy(host))
+                hp.copy_(torch.from_numpy(hsrc))
                 barrier()
                 t0 = time.perf_counter()
                 sb.solve_host_(hp)
@@ -294,10 +313,11 @@ def main():
             te = torch.tensor([float(np.mean(ts))], device="cuda", dtype=torch.float64)
             if ws > 1:
                 dist.all_reduce(te, op=dist.ReduceOp.MAX)
-            e2e = {"value": ws * B / float(te[0]), "unit": "RHS/s", "h2d_bytes_per_step": int(host.nbytes),
-                   "d2h_bytes_per_step": int(host.nbytes), "path": "spline_builder_solve_host (pinned, chunked)"}
+            e2e = {"value": ws * Be / float(te[0]), "unit": "RHS/s", "h2d_bytes_per_step": int(hsrc.nbytes),
+                   "d2h_bytes_per_step": int(hsrc.nbytes), "path": "spline_builder_solve_host (pinned, chunked)",
+                   "rhs_per_gpu": Be}
         else:
-            # point-contiguous: H2D copy + solve + D2H copy on the current stream
+            hp = torch.from_numpy(hsrc.copy()).pin_memory()
             dev = torch.empty_like(pristine)
             ts = []
             for _ in range(args.e2e_steps + 1):
@@ -308,8 +328,9 @@ def main():
                 hp.copy_(dev, non_blocking=True)
                 torch.cuda.synchronize()
                 ts.append(time.perf_counter() - t0)
-            e2e = {"value": ws * B / float(np.mean(ts[1:])), "unit": "RHS/s", "h2d_bytes_per_step": int(host.nbytes),
-                   "d2h_bytes_per_step": int(host.nbytes), "path": "H2D + spline_builder_solve + D2H"}
+            e2e = {"value": ws * B / float(np.mean(ts[1:])), "unit": "RHS/s", "h2d_bytes_per_step": int(hsrc.nbytes),
+                   "d2h_bytes_per_step": int(hsrc.nbytes), "path": "H2D + spline_builder_solve + D2H",
+                   "rhs_per_gpu": B}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
@@ -319,12 +340,14 @@ def main():
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "RHS/s", "n_gpus": ws, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong" if strong else "weak",
             "vs_baseline": None, "dtype": dt, "data": "synthetic (Philox U(-1,1) RHS, seeded)",
-            "config": {"workload": desc, "n": n, "batch_per_gpu": B, "degree": deg, "bc": ["periodic", "greville",
-                                                                                        "hermite"][bc],
+            "config": {"workload": desc, "n": n, "batch_per_gpu": B, "batch_total": B_total, "degree": deg,
+                       "bc": ["periodic", "greville", "hermite"][bc],
                        "mesh": mesh, "layout": "batch-contiguous" if layout == "batch" else "point-contiguous",
-                       "l2": f"inputs {host.nbytes / 1e6:.0f} MB per GPU > 126 MB L2; input restored + 256 MB L2 flush every 40 steps (untimed)",
+                       "l2": f"inputs {n * B * esz / 1e6:.0f} MB per GPU > 126 MB L2; input restored + 256 MB "
+                             f"L2 flush every 40 steps (untimed)",
+                       "inputs": "device Philox (inputs.rhs_device)" if on_device else "host Philox (inputs.rhs)",
                        "parallelism": f"dp{ws} (RHS shards)"},
             "achieved_gbs": achieved, "pct_of_8tbs": achieved / 8000.0,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

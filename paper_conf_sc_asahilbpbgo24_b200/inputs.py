@@ -83,6 +83,27 @@ def rhs(n: int, batch: int, seed: int = 1234, dtype=np.float64, degree: int = 3,
     return np.ascontiguousarray(b.astype(dtype))
 
 
+def rhs_device(n: int, batch: int, seed: int = 1234, first: int = 0, dtype=None, device="cuda",
+               out=None):
+    """Device-side twin of :func:`rhs` for batches too large for the host
+    (C5: 8e6 RHS = 64 GB).  Same block structure: block q of RHS_BLOCK
+    columns is U(-1, 1) from torch's CUDA Philox seeded with (seed, q), so a
+    shard [first, first+batch) holds exactly the columns of the unsharded
+    array.  (Values differ from the numpy generator of :func:`rhs`; parity
+    tests copy the sampled input columns to the host.)  Returns (n, batch)."""
+    import torch
+    dtype = dtype or torch.float64
+    x = out if out is not None else torch.empty((n, batch), dtype=dtype, device=device)
+    g = torch.Generator(device=device)
+    q0, q1 = first // RHS_BLOCK, (first + batch + RHS_BLOCK - 1) // RHS_BLOCK
+    for q in range(q0, q1):
+        g.manual_seed((seed * 1_000_003 + q) & 0x7FFFFFFFFFFFFFFF)
+        blk = torch.rand((n, RHS_BLOCK), generator=g, dtype=torch.float64, device=device).mul_(2.0).sub_(1.0)
+        lo, hi = max(first, q * RHS_BLOCK), min(first + batch, (q + 1) * RHS_BLOCK)
+        x[:, lo - first:hi - first].copy_(blk[:, lo - q * RHS_BLOCK:hi - q * RHS_BLOCK])
+    return x
+
+
 def gysela_slice(ny: int = 64, nv: int = 64, nmu: int = 32, nx: int = 1024, seed: int = 7,
                  dtype=np.float64) -> np.ndarray:
     """f[y][v][mu][x], x contiguous."""

@@ -184,3 +184,30 @@ def test_c3_full_size_sampled(torch_cuda, bc, npts):
     ref = o.solve(np.ascontiguousarray(b[:, idx]))
     assert rel_coef_error(got[:, idx], ref) <= TOL64
     assert o.residual(got[:, idx], b[:, idx]) <= TOL64
+
+
+def test_c5_shards_bitwise_equal_and_sampled_parity(torch_cuda):
+    """C5 recipe: device-generated RHS (inputs.rhs_device), sharded into
+    contiguous slices; each shard solved on its own equals the unsharded solve
+    bit for bit (per-RHS arithmetic is independent of the shard), and a seeded
+    sample matches the oracle."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200.shard import shard_bounds
+    sb, o = make(3, 1000, PERIODIC, "uniform")
+    total = 20000
+    full = inputs.rhs_device(sb.n, total, seed=99)
+    b_host = full.cpu().numpy()
+    sb.solve_(full)
+    for world in (2, 3):
+        parts = []
+        for rank in range(world):
+            a, b = shard_bounds(rank, world, total)
+            x = inputs.rhs_device(sb.n, b - a, seed=99, first=a)
+            assert torch.equal(x.cpu(), torch.from_numpy(b_host[:, a:b]))
+            sb.solve_(x)
+            parts.append(x)
+        assert torch.equal(torch.cat(parts, dim=1), full)
+    torch.cuda.synchronize()
+    idx = np.unique(np.concatenate([[0, total - 1], np.random.default_rng(5).choice(total, 512, replace=False)]))
+    got = full.cpu().numpy()[:, idx]
+    assert rel_coef_error(got, o.solve(np.ascontiguousarray(b_host[:, idx]))) <= TOL64
