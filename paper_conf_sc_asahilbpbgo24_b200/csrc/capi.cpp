@@ -71,7 +71,7 @@ int upload(spline_builder *h) {
     for (int d = 0; d < k; ++d) dscale[d] = P.rowscale[P.drow[d]];
     Packer pk;
     // per segment plan: factor arrays in the padded per-segment layout of device.hpp
-    struct SegOff { size_t L[2], U[2], D[2], G[2], H[2], gptr; int LP; };
+    struct SegOff { size_t L[2], U[2], D[2], G[2], H[2], gptr, slot; int LP, nslots; };
     SegOff so[3];
     for (int g = 0; g < 3; ++g) {
         const sb::SegPlan &G = P.seg[g];
@@ -80,17 +80,46 @@ int upload(spline_builder *h) {
         const int LP = g == 0 ? G.L + 2 : (g == 1 ? G.L + 4 : G.L);
         so[g].LP = LP;
         const int S = G.S;
-        std::vector<double> Lr((size_t)K * S * LP, 0.0), Ur((size_t)K * S * LP, 0.0), dinv((size_t)S * LP, 1.0);
-        for (int s = 0; s < S; ++s)
+        // factor data of each segment (identity on padding rows); segments with
+        // bitwise-identical data share one storage slot, so lanes reading them
+        // broadcast (uniform meshes: the LDL^T factors converge after ~30 rows)
+        std::vector<std::vector<double>> segdata(S);
+        for (int s = 0; s < S; ++s) {
+            std::vector<double> &dsd = segdata[s];
+            dsd.assign((size_t)(2 * K + 1) * G.L, 0.0);
             for (int i = 0; i < G.L; ++i) {
                 const int row = s * G.L + i;
-                if (row >= nQ) continue;  // padding rows: identity
+                dsd[(size_t)2 * K * G.L + i] = 1.0;
+                if (row >= nQ) continue;
                 for (int m = 0; m < K; ++m) {
-                    Lr[((size_t)m * S + s) * LP + i] = P.Lb[(size_t)row * K + m];
-                    Ur[((size_t)m * S + s) * LP + i] = P.Ub[(size_t)row * K + m];
+                    dsd[(size_t)m * G.L + i] = P.Lb[(size_t)row * K + m];
+                    dsd[(size_t)(K + m) * G.L + i] = P.Ub[(size_t)row * K + m];
                 }
-                dinv[(size_t)s * LP + i] = P.dinv[row];
+                dsd[(size_t)2 * K * G.L + i] = P.dinv[row];
             }
+        }
+        std::vector<int> slot(std::max(S, 1), 0), uniq;
+        for (int s = 0; s < S; ++s) {
+            int found = -1;
+            for (size_t u = 0; u < uniq.size() && found < 0; ++u)
+                if (segdata[uniq[u]] == segdata[s]) found = (int)u;
+            if (found < 0) { found = (int)uniq.size(); uniq.push_back(s); }
+            slot[s] = found;
+        }
+        const int NS = std::max(1, (int)uniq.size());
+        so[g].nslots = NS;
+        std::vector<double> Lr((size_t)K * NS * LP, 0.0), Ur((size_t)K * NS * LP, 0.0), dinv((size_t)NS * LP, 1.0);
+        for (size_t u = 0; u < uniq.size(); ++u) {
+            const std::vector<double> &dsd = segdata[uniq[u]];
+            for (int i = 0; i < G.L; ++i) {
+                for (int m = 0; m < K; ++m) {
+                    Lr[((size_t)m * NS + u) * LP + i] = dsd[(size_t)m * G.L + i];
+                    Ur[((size_t)m * NS + u) * LP + i] = dsd[(size_t)(K + m) * G.L + i];
+                }
+                dinv[u * LP + i] = dsd[(size_t)2 * K * G.L + i];
+            }
+        }
+        so[g].slot = pk.addv(slot);
         std::vector<int> gptr(S + 1, 0);
         for (int s = 0, e = 0; s <= S; ++s) {
             while (e < (int)P.gam_r.size() && P.gam_r[e] < s * G.L) ++e;
@@ -137,6 +166,7 @@ int upload(spline_builder *h) {
         const sb::SegPlan &G = P.seg[g];
         sb::DevSeg &ds = d.seg[g];
         ds.L = G.L; ds.S = G.S; ds.LP = so[g].LP; ds.carry_f = G.carry_f; ds.carry_b = G.carry_b;
+        ds.nslots = so[g].nslots; ds.slot = (const int *)at(so[g].slot);
         for (int c = 0; c < 2; ++c) {
             ds.Lr[c] = at(so[g].L[c]); ds.Ur[c] = at(so[g].U[c]); ds.dinv[c] = at(so[g].D[c]);
             ds.G[c] = at(so[g].G[c]); ds.H[c] = at(so[g].H[c]);

@@ -9,12 +9,15 @@ namespace sb {
 // Segment plan of one kernel family: Q padded to S*L rows, split into S
 // register segments of L rows.  Factor arrays are stored per segment with a
 // padded pitch LP (bank-conflict-free broadcast reads, 16-B aligned pairs):
-//   L(a+i, a+i-1-m)  at Lr[(m*S + s)*LP + i]      (a = s*L)
-//   U'(a+i, a+i+1+m) at Ur[(m*S + s)*LP + i]
-//   dinv(a+i)        at dinv[s*LP + i]             (1 on padding rows)
+//   L(a+i, a+i-1-m)  at Lr[(m*NS + slot[s])*LP + i]      (a = s*L, NS = nslots)
+//   U'(a+i, a+i+1+m) at Ur[(m*NS + slot[s])*LP + i]
+//   dinv(a+i)        at dinv[slot[s]*LP + i]               (1 on padding rows)
+// Segments with bitwise-identical factors share a slot (broadcast reads).
 // Floating-point arrays exist in fp64 ([0]) and fp32 ([1]).
 struct DevSeg {
     int L, S, LP, carry_f, carry_b;
+    int nslots;               // distinct factor blocks; segment s reads block slot[s]
+    const int *slot;
     const void *Lr[2], *Ur[2], *dinv[2];
     const void *G[2], *H[2];  // S*K*K forward / backward segment transfer matrices
     const int *gptr;          // S+1: gamma COO entries of segment s are [gptr[s], gptr[s+1])

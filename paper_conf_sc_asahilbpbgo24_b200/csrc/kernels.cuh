@@ -60,6 +60,7 @@ struct KParams {
         off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, off_cbuf,
         smem_total;
     int wbuf_pitch;                  // warp kernel: elements per per-warp row buffer
+    int bulk, warp_threads;          // warp kernel: bulk-copy pipeline on/off, threads per block
 };
 
 // ------------------------------------------------------------- PTX helpers
@@ -263,11 +264,11 @@ __device__ __forceinline__ void stage_constants(const KParams &p, const DevSeg &
     constexpr int CI = sizeof(C) == 8 ? 0 : 1;
     const DevPlan &P = p.P;
     const int k = P.k, S = G.S;
-    const int nrec = K * S * G.LP;
+    const int nrec = K * G.nslots * G.LP;
     copy_words(reinterpret_cast<C *>(smem + p.off_L), reinterpret_cast<const C *>(G.Lr[CI]), nrec, tid, nthreads);
     copy_words(reinterpret_cast<C *>(smem + p.off_U), reinterpret_cast<const C *>(G.Ur[CI]), nrec, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_dinv), reinterpret_cast<const C *>(G.dinv[CI]), S * G.LP, tid,
-               nthreads);
+    copy_words(reinterpret_cast<C *>(smem + p.off_dinv), reinterpret_cast<const C *>(G.dinv[CI]), G.nslots * G.LP,
+               tid, nthreads);
     copy_words(reinterpret_cast<C *>(smem + p.off_G), reinterpret_cast<const C *>(G.G[CI]), S * K * K, tid, nthreads);
     copy_words(reinterpret_cast<C *>(smem + p.off_H), reinterpret_cast<const C *>(G.H[CI]), S * K * K, tid, nthreads);
     copy_words(reinterpret_cast<int *>(smem + p.off_lamptr), P.lam_ptr, k + 1, tid, nthreads);
@@ -314,7 +315,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int S = G.S, LP = G.LP, nQ = P.nQ, k = P.k, s_lo = P.s_lo;
     const int ncw = p.ncw, nbox = p.nbox, boxr = p.boxr;
-    const int ms = S * LP;  // band stride of the factor arrays
+    const int ms = G.nslots * LP;  // band stride of the factor arrays
 
     C *sL = reinterpret_cast<C *>(smem + p.off_L);
     C *sU = reinterpret_cast<C *>(smem + p.off_U);
@@ -448,7 +449,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const bool active = s < S;
     const int a = s * L;
     const bool full_seg = a + L <= nQ;
-    const int sc = active ? s : 0;  // idle threads of the last warp alias segment 0
+    const int sc = G.slot[active ? s : 0];  // factor block (idle threads alias segment 0)
     const C *fL = sL + (size_t)sc * LP;
     const C *fU = sU + (size_t)sc * LP;
     const C *fD = sdinv + (size_t)sc * LP;
@@ -622,18 +623,46 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
 
 // ========================================================= warp kernel
 // One warp per RHS; lane s owns segment s (rows [s*L, s*L+L) of Q).
-template <typename T, int K, int L>
+// BULK: rows are contiguous and 16-B aligned -- lane 0 moves a whole row with
+// one cp.async.bulk (global->smem, mbarrier complete_tx) into one of two
+// per-warp row buffers, so the next row streams in while this one is solved,
+// and writes the result back with one bulk smem->global copy.
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *mbar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(mbar))
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_store(void *dst, const void *src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+template <typename T, int K, int L, bool BULK>
 __global__ void __launch_bounds__(256)
     sb_warp_kernel(const __grid_constant__ KParams p) {
     using C = T;
-    constexpr int CI = sizeof(T) == 8 ? 0 : 1;
     extern __shared__ __align__(1024) unsigned char smem[];
     const DevPlan &P = p.P;
     const DevSeg &G = P.seg[2];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int S = G.S, LP = G.LP, nQ = P.nQ, k = P.k, s_lo = P.s_lo, n = P.n;
-    const int ms = S * LP;
+    const int ms = G.nslots * LP;
+    const int nwarps = blockDim.x >> 5;
 
+    uint64_t *wbar = reinterpret_cast<uint64_t *>(smem + p.off_mbar) + 2 * warp;  // 2 per warp
+    if (BULK && lane == 0) {
+        mbar_init(wbar, 1);
+        mbar_init(wbar + 1, 1);
+        fence_mbar_init();
+    }
     stage_constants<C, K>(p, G, smem, tid, blockDim.x);
     __syncthreads();
 
@@ -652,39 +681,51 @@ __global__ void __launch_bounds__(256)
     const int *sdpiv = reinterpret_cast<const int *>(smem + p.off_dpiv);
     const C *sdscale = reinterpret_cast<const C *>(smem + p.off_dscale);
     const int *sdrow = reinterpret_cast<const int *>(smem + p.off_drow);
-    C *rowbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * p.wbuf_pitch;  // n values + k spare
-    C *x1 = rowbuf + n;  // k values after the row
+    // per warp: row buffer(s) of n values + k spare for x1
+    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * (BULK ? 2 : 1) * p.wbuf_pitch;
 
     const int s = lane;
     const bool active = s < S;
     const int a = s * L;
-    const C *fL = sL + (size_t)(active ? s : 0) * LP;
-    const C *fU = sU + (size_t)(active ? s : 0) * LP;
-    const C *fD = sdinv + (size_t)(active ? s : 0) * LP;
+    const int slot = G.slot[active ? s : 0];  // identical segments share (and broadcast) one block
+    const C *fL = sL + (size_t)slot * LP;
+    const C *fU = sU + (size_t)slot * LP;
+    const C *fD = sdinv + (size_t)slot * LP;
     T *gout = reinterpret_cast<T *>(p.rhs);
     const int64_t ps = p.pstride;
     const bool vec = (ps == 1) && ((p.bstride * (int64_t)sizeof(T)) % 16 == 0) &&
                      ((uintptr_t)p.rhs % 16 == 0) && (n % (16 / (int)sizeof(T)) == 0);
     constexpr int VW = 16 / sizeof(T);  // elements per 16-B vector
+    using V = typename std::conditional<sizeof(T) == 8, double2, float4>::type;
+    const uint32_t row_bytes = (uint32_t)(n * sizeof(T));
 
-    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + warp;
-    const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t rhs = gw; rhs < p.batch; rhs += nw) {
-        T *g = gout + rhs * p.bstride;
-        // ---------- coalesced load of the whole row
-        if (vec) {
-            using V = typename std::conditional<sizeof(T) == 8, double2, float4>::type;
-            const V *gv = reinterpret_cast<const V *>(g);
-            for (int q = lane; q < n / VW; q += 32) {
-                const V w = __ldcs(gv + q);
-                const T *pw = reinterpret_cast<const T *>(&w);
-#pragma unroll
-                for (int e = 0; e < VW; ++e) rowbuf[q * VW + e] = (C)pw[e];
+    const int64_t gw = (int64_t)blockIdx.x * nwarps + warp;
+    const int64_t nw = (int64_t)gridDim.x * nwarps;
+    if (BULK && lane == 0)
+        for (int b = 0; b < 2; ++b) {
+            const int64_t r = gw + b * nw;
+            if (r < p.batch) {
+                mbar_arrive_expect_tx(wbar + b, row_bytes);
+                bulk_load(wbuf + (size_t)b * p.wbuf_pitch, gout + r * p.bstride, row_bytes, wbar + b);
             }
-        } else {
-            for (int j = lane; j < n; j += 32) rowbuf[j] = (C)__ldcs(g + (int64_t)j * ps);
         }
-        __syncwarp();
+    int j = 0;
+    for (int64_t rhs = gw; rhs < p.batch; rhs += nw, ++j) {
+        T *g = gout + rhs * p.bstride;
+        C *rowbuf = wbuf + (BULK ? (size_t)(j & 1) * p.wbuf_pitch : 0);
+        C *x1 = rowbuf + n;  // k values after the row
+        // ---------- the whole row into shared memory
+        if (BULK) {
+            mbar_wait(wbar + (j & 1), (j >> 1) & 1);
+        } else if (vec) {
+            const V *gv = reinterpret_cast<const V *>(g);
+            V *sv = reinterpret_cast<V *>(rowbuf);  // C == T: whole 16-B vectors, conflict-free
+            for (int q = lane; q < n / VW; q += 32) sv[q] = __ldcs(gv + q);
+            __syncwarp();
+        } else {
+            for (int q = lane; q < n; q += 32) rowbuf[q] = (C)__ldcs(g + (int64_t)q * ps);
+            __syncwarp();
+        }
         // ---------- corner: x1 = delta'^{-1} (s1*b1 - Lambda b0), then b0 -= gamma x1
         if (k > 0) {
             for (int d = 0; d < k; ++d) {
@@ -751,26 +792,36 @@ __global__ void __launch_bounds__(256)
             }
             if (active && s < S - 1) bwd_correct<C, K, L, 1, false>(v, fU, ms, co);
         }
-        // ---------- back to the row buffer, coalesced store
+        // ---------- back to the row buffer, then to HBM
 #pragma unroll
         for (int i = 0; i < L; ++i)
             if (active && a + i < nQ) rowbuf[s_lo + a + i] = v[i][0];
-        __syncwarp();
-        if (vec) {
-            using V = typename std::conditional<sizeof(T) == 8, double2, float4>::type;
-            V *gv = reinterpret_cast<V *>(g);
-            for (int q = lane; q < n / VW; q += 32) {
-                V w;
-                T *pw = reinterpret_cast<T *>(&w);
-#pragma unroll
-                for (int e = 0; e < VW; ++e) pw[e] = (T)rowbuf[q * VW + e];
-                __stcs(gv + q, w);
+        if (BULK) {
+            fence_proxy_async_smem();  // generic smem writes -> visible to the bulk copy
+            __syncwarp();
+            if (lane == 0) {
+                bulk_store(g, rowbuf, row_bytes);
+                const int64_t nr = rhs + 2 * nw;  // next row for this buffer
+                if (nr < p.batch) {
+                    bulk_wait_read();  // the store has read the buffer
+                    mbar_arrive_expect_tx(wbar + (j & 1), row_bytes);
+                    bulk_load(rowbuf, gout + nr * p.bstride, row_bytes, wbar + (j & 1));
+                }
             }
+            __syncwarp();
+        } else if (vec) {
+            __syncwarp();
+            V *gv = reinterpret_cast<V *>(g);
+            const V *sv = reinterpret_cast<const V *>(rowbuf);
+            for (int q = lane; q < n / VW; q += 32) __stcs(gv + q, sv[q]);
+            __syncwarp();
         } else {
-            for (int j = lane; j < n; j += 32) __stcs(g + (int64_t)j * ps, (T)rowbuf[j]);
+            __syncwarp();
+            for (int q = lane; q < n; q += 32) __stcs(g + (int64_t)q * ps, (T)rowbuf[q]);
+            __syncwarp();
         }
-        __syncwarp();
     }
+    if (BULK && lane == 0) bulk_wait_all();
 }
 
 }  // namespace sb
@@ -818,10 +869,10 @@ int tile_K(int K, const KParams &kp, const CUtensorMap *tm, int grid, int thread
 
 template <typename T, int K, int L>
 int launch_warp1(const KParams &kp, int grid, cudaStream_t st, char *err, int errlen) {
-    auto fn = sb_warp_kernel<T, K, L>;
+    auto fn = kp.bulk ? sb_warp_kernel<T, K, L, true> : sb_warp_kernel<T, K, L, false>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total) != cudaSuccess)
         return check_launch("cudaFuncSetAttribute(warp)", err, errlen);
-    fn<<<grid, 256, kp.smem_total, st>>>(kp);
+    fn<<<grid, kp.warp_threads, kp.smem_total, st>>>(kp);
     return check_launch("warp kernel launch", err, errlen);
 }
 

@@ -35,9 +35,9 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     };
     const int K = P.K, k = P.k, S = G.S;
     kp.off_buf = take(buf_bytes, 1024);
-    kp.off_L = take((size_t)K * S * G.LP * esz, 16);
-    kp.off_U = take((size_t)K * S * G.LP * esz, 16);
-    kp.off_dinv = take((size_t)S * G.LP * esz, 16);
+    kp.off_L = take((size_t)K * G.nslots * G.LP * esz, 16);
+    kp.off_U = take((size_t)K * G.nslots * G.LP * esz, 16);
+    kp.off_dinv = take((size_t)G.nslots * G.LP * esz, 16);
     kp.off_G = take((size_t)S * K * K * esz, 16);
     kp.off_H = take((size_t)S * K * K * esz, 16);
     kp.off_fend = take((size_t)S * R * K * esz, 16);
@@ -74,14 +74,18 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
     kp.bstride = a.bstride;
     kp.pstride = a.pstride;
     kp.wbuf_pitch = (int)align_up((size_t)P.n + P.k + 2, 4);
-    layout_smem(kp, P, G, 1, esz, (size_t)8 * kp.wbuf_pitch * esz);
+    // bulk-copy pipeline when every row is one contiguous, 16-B aligned run
+    kp.bulk = a.pstride == 1 && (a.bstride * (int64_t)esz) % 16 == 0 && (uintptr_t)a.rhs % 16 == 0 &&
+              ((int64_t)P.n * (int64_t)esz) % 16 == 0;
+    const int wpb = kp.bulk ? 4 : 8;  // warps per block
+    kp.warp_threads = 32 * wpb;
+    layout_smem(kp, P, G, 1, esz, (size_t)wpb * (kp.bulk ? 2 : 1) * kp.wbuf_pitch * esz);
     if (kp.smem_total > max_smem) {
         snprintf(err, errlen, "warp kernel needs %d B of shared memory", kp.smem_total);
         return 5;
     }
-    const int per_sm = std::max(1, std::min(4, (int)(228 * 1024 / (kp.smem_total + 1024))));
-    const int64_t warps = (a.batch + 0);
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, (int64_t)num_sms * per_sm));
+    const int per_sm = std::max(1, std::min(8, (int)(228 * 1024 / (kp.smem_total + 1024))));
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + wpb - 1) / wpb, (int64_t)num_sms * per_sm));
     // round L up to an instantiated odd length (the plan chose the smallest odd L >= nQ/32)
     if (a.dtype == 0) return launch_warp_f64(P.K, G.L, kp, grid, a.stream, err, errlen);
     return launch_warp_f32(P.K, G.L, kp, grid, a.stream, err, errlen);
