@@ -26,6 +26,7 @@ SOURCES = [
     ("tile_f32.cu", "cu"),
     ("warp_f64.cu", "cu"),
     ("warp_f32.cu", "cu"),
+    ("serial.cu", "cu"),
 ]
 HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh"]
 

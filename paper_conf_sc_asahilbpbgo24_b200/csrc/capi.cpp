@@ -133,6 +133,15 @@ int upload(spline_builder *h) {
         so[g].H[0] = pk.addv(G.H); so[g].H[1] = pk.addv(conv<float>(G.H));
         so[g].gptr = pk.addv(gptr);
     }
+    std::vector<double> rowf((size_t)std::max(nQ, 1) * (2 * K + 1), 0.0);
+    for (int i = 0; i < nQ; ++i) {
+        for (int m = 0; m < K; ++m) {
+            rowf[(size_t)i * (2 * K + 1) + m] = P.Lb[(size_t)i * K + m];
+            rowf[(size_t)i * (2 * K + 1) + K + m] = P.Ub[(size_t)i * K + m];
+        }
+        rowf[(size_t)i * (2 * K + 1) + 2 * K] = P.dinv[i];
+    }
+    size_t oRowf[2] = {pk.addv(rowf), pk.addv(conv<float>(rowf))};
     size_t oLam[2], oGam[2], oDlu[2], oDs[2];
     for (int c = 0; c < 2; ++c) {
         auto put = [&](const std::vector<double> &v) { return c == 0 ? pk.addv(v) : pk.addv(conv<float>(v)); };
@@ -161,6 +170,7 @@ int upload(spline_builder *h) {
     }
     for (int c = 0; c < 2; ++c) {
         d.lam_v[c] = at(oLam[c]); d.gam_v[c] = at(oGam[c]); d.dlu[c] = at(oDlu[c]); d.dscale[c] = at(oDs[c]);
+        d.rowf[c] = at(oRowf[c]);
     }
     for (int g = 0; g < 3; ++g) {
         const sb::SegPlan &G = P.seg[g];

@@ -30,6 +30,7 @@ struct DevPlan {
     int lam_nnz, gam_nnz;    // Lambda CSR / gamma COO sizes
     int corner_rows;         // rows [0,c) and [n-c,n) hold every row the corner reads (0: none/unbounded)
     const void *lam_v[2], *gam_v[2], *dlu[2], *dscale[2];
+    const void *rowf[2];     // nQ x (2K+1): L(i,i-1..i-K), U'(i,i+1..i+K), dinv(i) -- serial fallback
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
     DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),
                              // [2] warp-per-RHS kernel (odd L; S == 0 if unavailable)

@@ -824,6 +824,71 @@ __global__ void __launch_bounds__(256)
     if (BULK && lane == 0) bulk_wait_all();
 }
 
+// ========================================================= serial fallback
+// One thread per RHS walks all n rows in global memory (the paper's fused
+// Listing 6 structure): any n, any strides.  Used only when the
+// register-segment kernels do not apply (Q longer than 32 x 63 rows).
+template <typename T, int K>
+__global__ void __launch_bounds__(128)
+    sb_serial_kernel(const __grid_constant__ KParams p) {
+    using C = T;
+    constexpr int CI = sizeof(T) == 8 ? 0 : 1;
+    constexpr int RW = 2 * K + 1;
+    const DevPlan &P = p.P;
+    const int nQ = P.nQ, k = P.k, s_lo = P.s_lo;
+    const C *rowf = reinterpret_cast<const C *>(P.rowf[CI]);
+    const C *lamv = reinterpret_cast<const C *>(P.lam_v[CI]);
+    const C *gamv = reinterpret_cast<const C *>(P.gam_v[CI]);
+    const C *dlu = reinterpret_cast<const C *>(P.dlu[CI]);
+    const C *dscale = reinterpret_cast<const C *>(P.dscale[CI]);
+    T *gout = reinterpret_cast<T *>(p.rhs);
+    const int64_t ps = p.pstride;
+    C x1[32];
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < p.batch; r += (int64_t)gridDim.x * blockDim.x) {
+        T *g = gout + r * p.bstride;
+        T *q0 = g + (int64_t)s_lo * ps;
+        // corner: x1 = delta'^-1 (s1 b1 - Lambda b0);  b0 -= gamma x1
+        for (int d = 0; d < k; ++d) {
+            C acc = (C)g[(int64_t)P.drow[d] * ps] * dscale[d];
+            for (int e = P.lam_ptr[d]; e < P.lam_ptr[d + 1]; ++e) acc = fma(-lamv[e], (C)q0[(int64_t)P.lam_c[e] * ps], acc);
+            x1[d] = acc;
+        }
+        if (k > 0) getrs_small(x1, dlu, P.dpiv, k);
+        for (int e = 0; e < P.gam_nnz; ++e) {
+            T *q = q0 + (int64_t)P.gam_r[e] * ps;
+            *q = (T)((C)*q - gamv[e] * x1[P.gam_c[e]]);
+        }
+        // forward sweep in place: y_i = b_i - sum_m L(i,i-1-m) y_{i-1-m}
+        C st[K];
+#pragma unroll
+        for (int m = 0; m < K; ++m) st[m] = C(0);
+        for (int i = 0; i < nQ; ++i) {
+            const C *f = rowf + (size_t)i * RW;
+            C acc = (C)q0[(int64_t)i * ps];
+#pragma unroll
+            for (int m = K - 1; m >= 0; --m) acc = fma(-__ldg(f + m), st[m], acc);
+#pragma unroll
+            for (int m = K - 1; m > 0; --m) st[m] = st[m - 1];
+            st[0] = acc;
+            q0[(int64_t)i * ps] = (T)acc;
+        }
+        // backward sweep in place: x_i = y_i dinv_i - sum_m U'(i,i+1+m) x_{i+1+m}
+#pragma unroll
+        for (int m = 0; m < K; ++m) st[m] = C(0);
+        for (int i = nQ - 1; i >= 0; --i) {
+            const C *f = rowf + (size_t)i * RW;
+            C acc = (C)q0[(int64_t)i * ps] * __ldg(f + 2 * K);
+#pragma unroll
+            for (int m = K - 1; m >= 0; --m) acc = fma(-__ldg(f + K + m), st[m], acc);
+#pragma unroll
+            for (int m = K - 1; m > 0; --m) st[m] = st[m - 1];
+            st[0] = acc;
+            q0[(int64_t)i * ps] = (T)acc;
+        }
+        for (int d = 0; d < k; ++d) g[(int64_t)P.drow[d] * ps] = (T)x1[d];
+    }
+}
+
 }  // namespace sb
 
 namespace sb {
@@ -834,6 +899,7 @@ int launch_tile_f32(int R, int loader, int K, const KParams &kp, const CUtensorM
                     cudaStream_t st, char *err, int errlen);
 int launch_warp_f64(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 int launch_warp_f32(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
+int launch_serial(int dtype, int K, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 
 inline int check_launch(const char *what, char *err, int errlen) {
     cudaError_t e = cudaGetLastError();

@@ -63,9 +63,15 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
 int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem, char *err, int errlen) {
     const size_t esz = a.dtype == 0 ? 8 : 4;
     const DevSeg &G = P.seg[2];
-    if (G.S == 0) {
-        snprintf(err, errlen, "n=%d too large for the warp-per-RHS kernel", P.n);
-        return 5;
+    if (G.S == 0) {  // Q too long for 32 register segments: serial fallback
+        KParams kp{};
+        kp.P = P;
+        kp.rhs = a.rhs;
+        kp.batch = a.batch;
+        kp.bstride = a.bstride;
+        kp.pstride = a.pstride;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
+        return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
     }
     KParams kp{};
     kp.P = P;
@@ -74,16 +80,25 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
     kp.bstride = a.bstride;
     kp.pstride = a.pstride;
     kp.wbuf_pitch = (int)align_up((size_t)P.n + P.k + 2, 4);
-    // bulk-copy pipeline when every row is one contiguous, 16-B aligned run
-    kp.bulk = a.pstride == 1 && (a.bstride * (int64_t)esz) % 16 == 0 && (uintptr_t)a.rhs % 16 == 0 &&
-              ((int64_t)P.n * (int64_t)esz) % 16 == 0;
-    const int wpb = kp.bulk ? 4 : 8;  // warps per block
-    kp.warp_threads = 32 * wpb;
-    layout_smem(kp, P, G, 1, esz, (size_t)wpb * (kp.bulk ? 2 : 1) * kp.wbuf_pitch * esz);
-    if (kp.smem_total > max_smem) {
-        snprintf(err, errlen, "warp kernel needs %d B of shared memory", kp.smem_total);
-        return 5;
+    // bulk-copy pipeline when every row is one contiguous, 16-B aligned run;
+    // fewer warps per block (or no second buffer) when shared memory is short
+    const bool can_bulk = a.pstride == 1 && (a.bstride * (int64_t)esz) % 16 == 0 && (uintptr_t)a.rhs % 16 == 0 &&
+                          ((int64_t)P.n * (int64_t)esz) % 16 == 0;
+    bool fits = false;
+    for (int cfg = 0; cfg < 6 && !fits; ++cfg) {
+        const bool bulk = cfg < 3 && can_bulk;
+        const int wpb = (cfg % 3 == 0) ? (bulk ? 4 : 8) : (cfg % 3 == 1 ? 2 : 1);
+        if (cfg < 3 && !can_bulk) continue;
+        kp.bulk = bulk;
+        kp.warp_threads = 32 * wpb;
+        layout_smem(kp, P, G, 1, esz, (size_t)wpb * (bulk ? 2 : 1) * kp.wbuf_pitch * esz);
+        fits = kp.smem_total <= max_smem;
     }
+    if (!fits) {  // factors + one row do not fit: serial fallback
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
+        return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
+    }
+    const int wpb = kp.warp_threads / 32;
     const int per_sm = std::max(1, std::min(8, (int)(228 * 1024 / (kp.smem_total + 1024))));
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + wpb - 1) / wpb, (int64_t)num_sms * per_sm));
     // round L up to an instantiated odd length (the plan chose the smallest odd L >= nQ/32)

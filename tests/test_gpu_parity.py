@@ -211,3 +211,21 @@ def test_c5_shards_bitwise_equal_and_sampled_parity(torch_cuda):
     idx = np.unique(np.concatenate([[0, total - 1], np.random.default_rng(5).choice(total, 512, replace=False)]))
     got = full.cpu().numpy()[:, idx]
     assert rel_coef_error(got, o.solve(np.ascontiguousarray(b_host[:, idx]))) <= TOL64
+
+
+@pytest.mark.parametrize("n_points,bc,p", [(1500, PERIODIC, 3), (2000, GREVILLE, 5), (3000, PERIODIC, 3),
+                                           (4100, HERMITE, 5)])
+@pytest.mark.parametrize("layout", ["batch", "point"])
+def test_large_n_paths(torch_cuda, n_points, bc, p, layout):
+    """n beyond the 1-CTA tile: R=8 tiles, the warp kernel with L=63, and the
+    serial fallback (one thread per RHS) for Q longer than 32 x 63 rows."""
+    torch = torch_cuda
+    sb, o = make(p, n_points, bc, "sin")
+    b = inputs.rhs(sb.n, 70, seed=21, degree=p, bc=bc)
+    ref = o.solve(b)
+    t = torch.from_numpy(b if layout == "batch" else np.ascontiguousarray(b.T)).cuda()
+    sb.solve_(t)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    got = got if layout == "batch" else got.T
+    assert rel_coef_error(got, ref) <= TOL64
