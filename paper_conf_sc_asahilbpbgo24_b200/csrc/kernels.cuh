@@ -353,8 +353,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             mbar_init(full + c, 1);
             mbar_init(empty + c, p.empty_count[c]);
         }
-        mbar_init(x1full + 0, 1);
-        mbar_init(x1full + 1, 1);
+        mbar_init(x1full + 0, R);  // every x1-writing corner lane arrives (release of its own writes)
+        mbar_init(x1full + 1, R);
         mbar_init(cfull + 0, 1);
         mbar_init(cfull + 1, 1);
         fence_mbar_init();
@@ -431,8 +431,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                     for (int d = 0; d < k; ++d) __stcs(gout + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
             }
             __syncwarp();
+            if (part == 0) mbar_arrive(x1full + (it & 1));
             if (lane == 0) {
-                mbar_arrive(x1full + (it & 1));
                 if (LOADER == LOAD_TMA)
                     for (int c = 0; c < nbox; ++c)
                         if (!use_cbox || ((p.corner_arrive_mask >> c) & 1)) mbar_arrive(empty + c);
