@@ -55,6 +55,7 @@ def _load():
         lib.oracle_get_rows.argtypes = [vp, dp, dp, dp]
         lib.oracle_handle_solve.argtypes = [vp, dp, i64, i64, i64, i32]
         lib.oracle_eval.argtypes = [vp, dp, i32, dp, i64, dp]
+        lib.oracle_advect.argtypes = [vp, dp, i64, i64, i64, dp, i32]
         _lib = lib
     return _lib
 
@@ -130,6 +131,17 @@ class Oracle:
         xs = np.ascontiguousarray(xs, dtype=np.float64)
         out = np.empty(xs.shape[0], dtype=np.float64)
         _lib.oracle_eval(self._h, _ptr(coef), int(deriv), _ptr(xs), int(xs.shape[0]), _ptr(out))
+        return out
+
+    def advect(self, f: np.ndarray, shift: np.ndarray, nthreads: int = 0) -> np.ndarray:
+        """One Algorithm-2 step on f of shape (n, batch)
+        (batch contiguous): spline build + evaluation at xi_i - shift[r]."""
+        out = np.array(f, dtype=np.float64, order="C", copy=True)
+        sh = np.ascontiguousarray(shift, dtype=np.float64)
+        assert out.ndim == 2 and out.shape[0] == self.n and sh.shape == (out.shape[1],)
+        st = _lib.oracle_advect(self._h, _ptr(out), int(out.shape[1]), 1, int(out.shape[1]), _ptr(sh), int(nthreads))
+        if st:
+            raise RuntimeError(f"oracle advect failed: {st}")
         return out
 
     def residual(self, x: np.ndarray, b: np.ndarray) -> float:

@@ -359,3 +359,56 @@ def test_oracle_bc_row_counts():
     assert Oracle(5, 1000, GREVILLE).n == 1000
     with pytest.raises(ValueError):
         Oracle(3, 10, GREVILLE, np.array([0.0, 0.5, 0.4, 1.0, 1.1, 1.2, 1.3, 1.4]))
+
+
+# ------------------------------------------------ advection step (NEXT f1)
+
+@pytest.mark.parametrize("p", [2, 3, 4, 5])
+def test_advect_integer_cell_shift_is_exact_roll(p):
+    """Algorithm 2 on a uniform periodic mesh: shifting by m whole
+    cells maps the spline space onto itself, so f_new = roll(f, m) exactly."""
+    N = 64
+    o = Oracle(p, N, PERIODIC)
+    f = rng(11).uniform(-1, 1, size=(N, 3))
+    h = 1.0 / N
+    for m in (0, 1, 5, -3):
+        out = o.advect(f, np.full(3, m * h))
+        assert np.abs(out - np.roll(f, m, axis=0)).max() < 1e-13
+
+
+@pytest.mark.parametrize("p", [3, 5])
+@pytest.mark.parametrize("kind", ["uniform", "jitter"])
+def test_advect_matches_scipy_spline_evaluation(p, kind):
+    """fractional shifts: the oracle's evaluation equals scipy's BSpline of the
+    same coefficients at the feet of the characteristics."""
+    N = 40
+    x = mesh(N, kind)
+    o = Oracle(p, N, PERIODIC, None if kind == "uniform" else x)
+    f = rng(12).uniform(-1, 1, size=(N, 4))
+    shift = np.array([0.0123, -0.37, 0.5, 1.77])
+    out = o.advect(f, shift)
+    c = o.solve(f)
+    g, t = periodic_ext_knots(x, p)
+    s = (p + 1) // 2
+    pts, _, _ = o.rows()
+    for r in range(4):
+        # our basis j has first knot j-s; scipy's BSpline(t, c', p) basis i has first knot t[i]
+        off = -g[0]
+        cext = np.zeros(len(t) - p - 1)
+        for j in range(-2 * N, 3 * N):
+            i = off + j - s
+            if 0 <= i < len(cext):
+                cext[i] = c[j % N, r]
+        spl = si.BSpline(t, cext, p, extrapolate=False)
+        feet = np.mod(pts - shift[r], 1.0)
+        assert np.abs(spl(feet) - out[:, r]).max() < 1e-12
+
+
+def test_advect_smooth_profile_is_accurate():
+    """a smooth periodic profile is transported to ~h^4 accuracy (cubic)."""
+    N = 128
+    o = Oracle(3, N, PERIODIC)
+    xs = np.arange(N) / N
+    f = np.sin(2 * np.pi * xs)[:, None]
+    out = o.advect(f, np.array([0.2345]))
+    assert np.abs(out[:, 0] - np.sin(2 * np.pi * (xs - 0.2345))).max() < 1e-6
