@@ -35,7 +35,9 @@ sys.path.insert(0, ROOT)
 from paper_conf_sc_asahilbpbgo24_b200 import inputs  # noqa: E402
 
 METRIC = "RHS/s and achieved HBM GB/s (% of peak), cubic n=1000, 1e5 RHS, fp64"
+ADV_METRIC = "advection GLUPS (Eq. 7: Nx*Nv / step time), one Algorithm-2 step"
 STRONG = {"C5"}            # total batch fixed, sharded over the ranks
+ADVECT = {"ADV", "ADVNU"}  # one semi-Lagrangian step (Algorithm 2) per step, metric GLUPS (Eq. 7)
 DEVICE_INPUT_ELEMS = 4e8   # above this, inputs are generated on the device (inputs.rhs_device)
 E2E_MAX_RHS = 1_000_000    # the e2e leg moves at most this many RHS through host memory
 
@@ -50,6 +52,10 @@ WORKLOADS = {
            "C4 GYSELA slice f[64][64][32][x=1024] cubic periodic along x, x contiguous, fp64"),
     "C4F32": (3, 1024, 0, "uniform", 131072, "f32", "point",
               "C4 GYSELA slice f[64][64][32][x=1024] cubic periodic along x, x contiguous, fp32"),
+    "ADV": (3, 1024, 0, "uniform", 100000, "f64", "point",
+            "Algorithm 2 advection step: Nx=1024, Nv=1e5, cubic uniform periodic, x contiguous, fp64 (GLUPS)"),
+    "ADVNU": (3, 1024, 0, "sin", 100000, "f64", "point",
+              "Algorithm 2 advection step: Nx=1024, Nv=1e5, cubic non-uniform (sin map) periodic, fp64 (GLUPS)"),
     "C5": (3, 1000, 0, "uniform", 8000000, "f64", "batch",
            "C5 cubic uniform periodic n=1000, 8e6 RHS in total sharded over the GPUs (strong scaling) fp64"),
 }
@@ -146,25 +152,41 @@ def make_rhs(deg, n, bc, B, first, layout, dtype):
     return np.ascontiguousarray(b.astype(np.float32 if dtype == "f32" else np.float64))
 
 
-def cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0, max_rhs=None):
+def adv_shift(n_cells, B, first=0):
+    """Displacements of the advection workloads: shift_j = dt * v_j with v_j
+    on a uniform velocity grid in [-vmax, vmax), dt chosen so |shift| <= 2.5
+    cells (a CFL number above 1, as semi-Lagrangian schemes allow)."""
+    j = np.arange(first, first + B, dtype=np.float64)
+    v = -1.0 + 2.0 * (j % 100000) / 100000.0
+    return v * (2.5 / n_cells)
+
+
+def cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0, max_rhs=None, adv=False):
     """Time the oracle as it stands on a bounded sample; returns (RHS/s,
-    threads, sample description)."""
+    threads, sample description).  adv: one Algorithm-2 step per RHS."""
     import oracle
     o = oracle.Oracle(deg, npts, bc, knots)
     threads = len(os.sched_getaffinity(0))
+
+    def run(b):
+        if adv:
+            o.advect(b, adv_shift(o.N, b.shape[1]), nthreads=threads)
+        else:
+            o.solve_(b, nthreads=threads)
     probe = 256
     b = inputs.rhs(n, probe, seed=99, degree=deg, bc=bc)
     t0 = time.perf_counter()
-    o.solve_(b.copy(), nthreads=threads)
+    run(b.copy())
     dt = time.perf_counter() - t0
     m = int(max(probe, min(target_s / max(dt, 1e-6) * probe, 200000)))
     if max_rhs:
         m = min(m, max_rhs)
     b = inputs.rhs(n, m, seed=98, degree=deg, bc=bc)
     t0 = time.perf_counter()
-    o.solve_(b, nthreads=threads)
+    run(b)
     dt = time.perf_counter() - t0
-    return m / dt, threads, f"{m} RHS of the same workload (n={n}), dense GEPP oracle, {threads} OpenMP threads"
+    what = "solve + evaluation at the feet (Algorithm 2)" if adv else "dense GEPP oracle"
+    return m / dt, threads, f"{m} RHS of the same workload (n={n}), {what}, {threads} OpenMP threads"
 
 
 def run_reference(args, wl):
@@ -178,30 +200,39 @@ def run_reference(args, wl):
     o = oracle.Oracle(deg, npts, bc, knots)
     threads = len(os.sched_getaffinity(0))
     # each step: a bounded sample sized so the whole run stays within minutes
-    rate0, _, _ = cpu_oracle_rate(deg, npts, bc, knots, n, target_s=2.0)
+    adv = args.workload in ADVECT
+    rate0, _, _ = cpu_oracle_rate(deg, npts, bc, knots, n, target_s=2.0, adv=adv)
     per_step = max(64, int(rate0 * min(4.0, 120.0 / max(1, args.steps + args.warmup))))  # whole run ~2 min
     b0 = inputs.rhs(n, per_step, seed=1234, degree=deg, bc=bc)
+    sh0 = adv_shift(o.N, per_step)
+
+    def run(b):
+        if adv:
+            o.advect(b, sh0, nthreads=threads)
+        else:
+            o.solve_(b, nthreads=threads)
     for _ in range(args.warmup):
-        o.solve_(b0.copy(), nthreads=threads)
+        run(b0.copy())
     times = []
     for _ in range(args.steps):
         b = b0.copy()
         t0 = time.perf_counter()
-        o.solve_(b, nthreads=threads)
+        run(b)
         times.append(time.perf_counter() - t0)
     t = float(np.mean(times))
     val = per_step / t
     esz = 4 if dt == "f32" else 8
+    metric, unit, scale = (ADV_METRIC, "GLUPS", n / 1e9) if adv else (METRIC, "RHS/s", 1.0)
     line = {
-        "impl": "reference", "metric": METRIC, "value": val, "unit": "RHS/s", "n_gpus": args.gpus,
+        "impl": "reference", "metric": metric, "value": val * scale, "unit": unit, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": dt, "data": "synthetic",
         "config": {"workload": desc, "n": n, "batch_per_step": per_step, "degree": deg, "bc": bc},
         "achieved_gbs": val * 2 * n * esz / 1e9,
-        "cpu_baseline": {"value": val, "unit": "RHS/s", "cores": threads, "kind": "oracle",
+        "cpu_baseline": {"value": val * scale, "unit": unit, "cores": threads, "kind": "oracle",
                          "sample": f"{per_step} RHS per step of the workload (n={n}); the full batch would take "
                                    f"{B / val:.1f} s"},
-        "e2e": {"value": val, "unit": "RHS/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "e2e": {"value": val * scale, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
@@ -252,6 +283,12 @@ def main():
         x = pristine.clone()
         restore = lambda: x.copy_(pristine)  # noqa: E731
     stream = torch.cuda.current_stream()
+    adv = args.workload in ADVECT
+    if adv:
+        shift = torch.from_numpy(adv_shift(inputs.n_cells(deg, npts, bc), B, first)).cuda()
+        step = lambda t: sb.advect_(t, shift)  # noqa: E731
+    else:
+        step = sb.solve_
 
     def barrier():
         if ws > 1:
@@ -264,7 +301,7 @@ def main():
     CHUNK = 40
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     for _ in range(args.warmup):
-        sb.solve_(x)
+        step(x)
     barrier()
     nchunks = (args.steps + CHUNK - 1) // CHUNK
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(nchunks)]
@@ -278,7 +315,7 @@ def main():
             flush.fill_(c & 0xFF)
             starts[c].record(stream)
             for _ in range(m):
-                sb.solve_(x)  # one fused kernel launch per step
+                step(x)  # one fused kernel launch per step
             ends[c].record(stream)
             done += m
         barrier()
@@ -324,22 +361,28 @@ def main():
                 barrier()
                 t0 = time.perf_counter()
                 dev.copy_(hp, non_blocking=True)
-                sb.solve_(dev)
+                step(dev)
                 hp.copy_(dev, non_blocking=True)
                 torch.cuda.synchronize()
                 ts.append(time.perf_counter() - t0)
-            e2e = {"value": ws * B / float(np.mean(ts[1:])), "unit": "RHS/s", "h2d_bytes_per_step": int(hsrc.nbytes),
-                   "d2h_bytes_per_step": int(hsrc.nbytes), "path": "H2D + spline_builder_solve + D2H",
+            te = torch.tensor([float(np.mean(ts[1:]))], device="cuda", dtype=torch.float64)
+            if ws > 1:
+                dist.all_reduce(te, op=dist.ReduceOp.MAX)
+            e2e = {"value": ws * B / float(te[0]) * (n / 1e9 if adv else 1.0), "unit": "GLUPS" if adv else "RHS/s",
+                   "h2d_bytes_per_step": int(hsrc.nbytes), "d2h_bytes_per_step": int(hsrc.nbytes),
+                   "path": "H2D + spline_builder_" + ("advect" if adv else "solve") + " + D2H",
                    "rhs_per_gpu": B}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
-        rate, cores, sample = cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0)
-        cpu = {"value": rate, "unit": "RHS/s", "cores": cores, "kind": "oracle", "sample": sample}
+        rate, cores, sample = cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0, adv=adv)
+        cpu = {"value": rate * (n / 1e9 if adv else 1.0), "unit": "GLUPS" if adv else "RHS/s", "cores": cores,
+               "kind": "oracle", "sample": sample}
 
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "RHS/s", "n_gpus": ws, "steps": args.steps,
+            "metric": ADV_METRIC if adv else METRIC, "value": value * (n / 1e9 if adv else 1.0),
+            "unit": "GLUPS" if adv else "RHS/s", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong" if strong else "weak",
             "vs_baseline": None, "dtype": dt, "data": "synthetic (Philox U(-1,1) RHS, seeded)",
             "config": {"workload": desc, "n": n, "batch_per_gpu": B, "batch_total": B_total, "degree": deg,

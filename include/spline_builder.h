@@ -114,6 +114,22 @@ int spline_builder_solve_strided(spline_builder_t h, void *rhs, int dtype, int64
                                  int64_t point_stride, void *stream);
 
 /*
+ * spline_builder_advect -- one step of the 1-D semi-Lagrangian advection of
+ * Algorithm 2 for a PERIODIC space, fused in one kernel:
+ * for every right-hand side r (one v_j line of f(x_i, v_j), same layout rules
+ * as spline_builder_solve_strided), the spline eta of f(., v_j) is built
+ * (Algorithm 1) and f is overwritten, in place, with eta evaluated at the feet
+ * of the characteristics:  f(xi_i, v_j) <- S_eta(xi_i - shift[r])  (periodic
+ * wrap), xi_i the interpolation points.  No transposes: the point-contiguous
+ * layout (batch_stride >= n, point_stride 1) is the fast path.
+ *   f      DEVICE pointer, SB_F64 or SB_F32 (dtype)
+ *   shift  DEVICE pointer to batch fp64 displacements (dt * v_j), in units of x
+ * Returns SB_UNSUPPORTED for non-periodic spaces.  Asynchronous on stream.
+ */
+int spline_builder_advect(spline_builder_t h, void *f, int dtype, int64_t batch, int64_t batch_stride,
+                          int64_t point_stride, const double *shift, void *stream);
+
+/*
  * spline_builder_solve_host -- end-to-end solve of HOST data (fp64 or fp32,
  * batch-contiguous (n, batch) layout with leading dimension ld >= batch):
  * the batch is cut into chunks that are copied host->device, solved and

@@ -129,6 +129,36 @@ class SplineBuilder:
                                                           _stream_handle(stream)))
         return rhs
 
+    def advect_(self, f, shift, batch_stride: int | None = None, stream=None):
+        """One semi-Lagrangian step of Algorithm 2, in
+        place: every RHS line of f (CUDA tensor, layouts as :meth:`solve_`) is
+        replaced by its spline evaluated at xi_i - shift[r] (periodic spaces).
+        ``shift``: CUDA fp64 tensor of batch displacements."""
+        import torch
+        if not (f.is_cuda and shift.is_cuda):
+            raise ValueError("f and shift must be CUDA tensors")
+        if shift.dtype != torch.float64 or not shift.is_contiguous():
+            raise TypeError("shift must be a contiguous float64 tensor")
+        if f.dim() != 2 or not f.is_contiguous():
+            raise ValueError("f must be a contiguous 2-D tensor")
+        if batch_stride is None:
+            if f.shape[0] == self.n:
+                batch, bs, pst = f.shape[1], 1, f.shape[1]
+            elif f.shape[1] == self.n:
+                batch, bs, pst = f.shape[0], self.n, 1
+            else:
+                raise ValueError(f"no dimension of size n={self.n}")
+        else:
+            bs = batch_stride
+            batch, pst = (f.shape[1], f.shape[1]) if bs == 1 else (f.shape[0], 1)
+        if shift.numel() != batch:
+            raise ValueError("shift must have one entry per right-hand side")
+        dt = SB_F64 if f.dtype == torch.float64 else SB_F32
+        _lib.check(self._lib.spline_builder_advect(self._h, ctypes.c_void_p(f.data_ptr()), dt, int(batch), int(bs),
+                                                   int(pst), ctypes.c_void_p(shift.data_ptr()),
+                                                   _stream_handle(stream)))
+        return f
+
     def solve_host_(self, arr, ld: int | None = None):
         """End-to-end solve of host memory (numpy array or CPU tensor of shape
         (n, >=batch), row-major).  Pinned memory gives full PCIe bandwidth."""

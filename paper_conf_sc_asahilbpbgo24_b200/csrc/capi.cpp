@@ -142,6 +142,7 @@ int upload(spline_builder *h) {
         rowf[(size_t)i * (2 * K + 1) + 2 * K] = P.dinv[i];
     }
     size_t oRowf[2] = {pk.addv(rowf), pk.addv(conv<float>(rowf))};
+    size_t oXe = pk.addv(P.xe), oXi = pk.addv(P.xi), oTbl = pk.addv(P.adv_tbl);
     size_t oLam[2], oGam[2], oDlu[2], oDs[2];
     for (int c = 0; c < 2; ++c) {
         auto put = [&](const std::vector<double> &v) { return c == 0 ? pk.addv(v) : pk.addv(conv<float>(v)); };
@@ -157,6 +158,7 @@ int upload(spline_builder *h) {
     auto at = [&](size_t off) { return (const void *)((const unsigned char *)h->blob + off); };
     sb::DevPlan &d = h->dp;
     d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K;
+    d.p = P.p; d.N = P.N; d.periodic = P.bc == sb::PERIODIC;
     d.lam_nnz = (int)P.Lam_v.size(); d.gam_nnz = (int)P.gam_v.size();
     {   // rows the corner step reads: delta rows (b1) and Lambda columns (b0)
         int head = 0, tail = 0;
@@ -183,6 +185,9 @@ int upload(spline_builder *h) {
         }
         ds.gptr = (const int *)at(so[g].gptr);
     }
+    d.xe = (const double *)at(oXe); d.xi = (const double *)at(oXi);
+    d.adv_uniform = P.adv_uniform ? 1 : 0; d.adv_invh = P.adv_invh; d.adv_q0 = P.adv_q0;
+    d.adv_tbl = (const int *)at(oTbl); d.adv_nbkt = (int)P.adv_tbl.size();
     d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
     d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);
     d.dpiv = (const int *)at(o_dpiv); d.drow = (const int *)at(o_drow);
@@ -190,7 +195,7 @@ int upload(spline_builder *h) {
 }
 
 int do_solve(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t bstride, int64_t pstride,
-             cudaStream_t stream) {
+             cudaStream_t stream, const double *shift = nullptr) {
     if (!h) return fail(SB_INVALID_ARG, "null handle");
     if (h->host_only) return fail(SB_UNSUPPORTED, "handle was created with SB_FLAG_HOST_ONLY");
     if (dtype != SB_F64 && dtype != SB_F32) return fail(SB_INVALID_ARG, "dtype must be SB_F64 or SB_F32");
@@ -206,7 +211,7 @@ int do_solve(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t bst
     int cur = -1;
     cudaGetDevice(&cur);
     if (cur != h->device) cudaSetDevice(h->device);
-    sb::SolveArgs a{rhs, batch, bstride, pstride, dtype, stream};
+    sb::SolveArgs a{rhs, batch, bstride, pstride, dtype, stream, shift};
     char err[256] = {0};
     int st = sb::launch_solve(h->dp, a, h->num_sms, err, sizeof(err));
     if (cur != h->device) cudaSetDevice(cur);
@@ -260,6 +265,14 @@ int spline_builder_solve_f32(spline_builder_t h, float *rhs, int64_t batch, int6
 int spline_builder_solve_strided(spline_builder_t h, void *rhs, int dtype, int64_t batch, int64_t batch_stride,
                                  int64_t point_stride, void *stream) {
     return do_solve(h, rhs, dtype, batch, batch_stride, point_stride, (cudaStream_t)stream);
+}
+
+int spline_builder_advect(spline_builder_t h, void *f, int dtype, int64_t batch, int64_t batch_stride,
+                          int64_t point_stride, const double *shift, void *stream) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (h->plan.bc != sb::PERIODIC) return fail(SB_UNSUPPORTED, "advect needs a periodic spline space");
+    if (batch > 0 && !shift) return fail(SB_INVALID_ARG, "shift is NULL");
+    return do_solve(h, f, dtype, batch, batch_stride, point_stride, (cudaStream_t)stream, shift);
 }
 
 int spline_builder_solve_host(spline_builder_t h, void *host_rhs, int dtype, int64_t batch, int64_t ld) {

@@ -31,6 +31,12 @@ struct DevPlan {
     int corner_rows;         // rows [0,c) and [n-c,n) hold every row the corner reads (0: none/unbounded)
     const void *lam_v[2], *gam_v[2], *dlu[2], *dscale[2];
     const void *rowf[2];     // nQ x (2K+1): L(i,i-1..i-K), U'(i,i+1..i+K), dinv(i) -- serial fallback
+    int p, N, periodic;      // spline degree, cells, periodic flag (advection / evaluation)
+    const double *xe, *xi;   // periodic extended knots t_c at xe[c+p] (N+2p+1), n row positions
+    int adv_uniform;         // uniform periodic mesh: Algorithm 2's evaluation is a per-row stencil
+    double adv_invh, adv_q0; // 1/h, (xi_0 - x_0)/h
+    const int *adv_tbl;      // non-uniform: bucket b of [x_0, x_N) in adv_nbkt -> cell of its left edge
+    int adv_nbkt;
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
     DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),
                              // [2] warp-per-RHS kernel (odd L; S == 0 if unavailable)
@@ -43,6 +49,7 @@ struct SolveArgs {
     int64_t pstride;   // elements between rows
     int dtype;         // 0 fp64, 1 fp32
     cudaStream_t stream;
+    const double *shift = nullptr;  // advect: per-RHS displacement (device, fp64); nullptr = plain solve
 };
 
 // returns 0 on success, else an SB_* status; fills err on failure

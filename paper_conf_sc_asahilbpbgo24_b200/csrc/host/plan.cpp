@@ -505,6 +505,40 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
             ++r;
         }
     }
+    // breakpoints and row positions (advection / evaluation data)
+    // (uniform: x_c = c/N on [0,1], not a running sum of widths, R1)
+    P.xb.assign(N + 1, 0.0);
+    for (int c = 0; c <= N; ++c) P.xb[c] = knots ? knots[c] : (double)c / (double)N;
+    P.xi.resize(n);
+    for (int i = 0; i < n; ++i) {
+        const long cell = bc == PERIODIC ? lmod(rows[i].span, N) : rows[i].span - p;
+        P.xi[i] = P.xb[cell] + rows[i].u;
+    }
+    if (bc == PERIODIC) {
+        // periodic extension t_c, c in [-p, N+p]: xe[c + p] (evaluation at the feet, Algorithm 2)
+        const double Lp = P.xb[N] - P.xb[0];
+        P.xe.resize(N + 2 * p + 1);
+        for (int c = -p; c <= N + p; ++c)
+            P.xe[c + p] = c < 0 ? P.xb[c + N] - Lp : (c > N ? P.xb[c - N] + Lp : P.xb[c]);
+        // uniform within one ulp: every foot of a row shares its local coordinate,
+        // so the evaluation is a (p+1)-tap stencil with weights computed once per row
+        const double hu = Lp / N;
+        double dev = 0.0, xmax = 1.0;
+        for (int c = 0; c <= N; ++c) {
+            dev = std::max(dev, std::fabs(P.xb[c] - (P.xb[0] + c * hu)));
+            xmax = std::max(xmax, std::fabs(P.xb[c]));
+        }
+        for (int i = 0; i < n; ++i) dev = std::max(dev, std::fabs((P.xi[i] - P.xi[0]) - i * hu));
+        P.adv_uniform = dev <= 2.3e-16 * xmax;
+        P.adv_invh = 1.0 / hu;
+        P.adv_q0 = (P.xi[0] - P.xb[0]) / hu;
+        P.adv_tbl.resize(2 * N);
+        for (int b = 0, c = 0; b < 2 * N; ++b) {
+            const double x = P.xb[0] + b * (Lp / (2.0 * N));
+            while (c + 1 < N && P.xb[c + 1] <= x) ++c;
+            P.adv_tbl[b] = c;
+        }
+    }
     // equilibrated sparse rows: rowscale * (d^deriv B_j)(point)
     P.A.assign(n, SparseRow());
     for (int i = 0; i < n; ++i) {

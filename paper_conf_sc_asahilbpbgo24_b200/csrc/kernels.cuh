@@ -61,6 +61,8 @@ struct KParams {
         smem_total;
     int wbuf_pitch;                  // warp kernel: elements per per-warp row buffer
     int bulk, warp_threads;          // warp kernel: bulk-copy pipeline on/off, threads per block
+    const double *shift;             // advect: per-RHS displacement (nullptr: plain solve)
+    int adv, off_geo;                // advect flag; smem offset of xb[N+1], hw[N], xi[n] (fp64)
 };
 
 // ------------------------------------------------------------- PTX helpers
@@ -645,7 +647,131 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
-template <typename T, int K, int L, bool BULK>
+// Algorithm 2's interpolation at the feet of the characteristics (PAPER.md
+// P:157-163): out[i] = S(xi_i - shift) for the periodic spline S with
+// coefficients coef[0..N) just solved for.  The p+1 nonzero B-splines at a
+// point come from de Boor's triangular scheme (BSPLVB) with
+// dl[j] = x - t_{c-j}, dr[j] = t_{c+1+j} - x; basis j of the centred periodic
+// space has its first knot at j - s, s = floor((p+1)/2), so the value is
+// sum_r b[r] coef[(c - p + r + s) mod N].
+template <int PD>
+__device__ __forceinline__ void bspl_values(const double (&dl)[PD], const double (&dr)[PD], double (&b)[PD + 1]) {
+    b[0] = 1.0;
+#pragma unroll
+    for (int j = 0; j < PD; ++j) {
+        double saved = 0.0;
+#pragma unroll
+        for (int r = 0; r <= j; ++r) {
+            const double term = b[r] / (dr[r] + dl[j - r]);
+            b[r] = saved + dr[r] * term;
+            saved = dl[j - r] * term;
+        }
+        b[j + 1] = saved;
+    }
+}
+
+// One row of the advection step.
+// Uniform mesh: every foot xi_i - shift has the same local coordinate u, so
+// the weights are computed once per row and out[i] = sum_r w_r coef[i+off+r]
+// is a (p+1)-tap stencil.  Lane l owns the run of window starts
+// [l*M, l*M+M) (M odd: conflict-free smem strides) and slides a register
+// window along it: ~N + 32p shared loads per row instead of (p+1) N.
+// Otherwise: per point, locate the cell through the bucket table, then
+// BSPLVB; U independent points per iteration for latency hiding.
+template <typename C, int PD>
+__device__ __forceinline__ void advect_row(const DevPlan &P, const double *sgeo, const C *coef, C *out, double sh,
+                                           int lane) {
+    constexpr int s = (PD + 1) / 2;
+    const int N = P.N;
+    if (P.adv_uniform) {
+        const double q = P.adv_q0 - sh * P.adv_invh;  // foot of point 0, in cells from x_0
+        const double cf = floor(q);
+        double dl[PD], dr[PD], b[PD + 1];
+#pragma unroll
+        for (int j = 0; j < PD; ++j) {
+            dl[j] = (q - cf) + j;
+            dr[j] = (j + 1) - (q - cf);
+        }
+        bspl_values<PD>(dl, dr, b);
+        C w[PD + 1];
+#pragma unroll
+        for (int r = 0; r <= PD; ++r) w[r] = (C)b[r];
+        int c0 = (int)(cf - (double)N * floor(cf / (double)N));
+        c0 = c0 >= N ? c0 - N : (c0 < 0 ? c0 + N : c0);
+        int off = c0 - PD + s;  // point i reads coef[i + off .. i + off + PD] (mod N)
+        off = off < 0 ? off + N : (off >= N ? off - N : off);
+        const int M = ((N + 31) >> 5) | 1;
+        const int cbeg = lane * M;
+        if (cbeg >= N) return;
+        const int cend = min(cbeg + M, N);
+        C win[PD + 1];
+        int idx = cbeg;
+#pragma unroll
+        for (int r = 0; r < PD; ++r) {
+            win[r] = coef[idx];
+            idx = idx + 1 == N ? 0 : idx + 1;
+        }
+        int jr = cbeg - off;
+        jr = jr < 0 ? jr + N : jr;
+        for (int c = cbeg; c < cend; ++c) {
+            win[PD] = coef[idx];
+            idx = idx + 1 == N ? 0 : idx + 1;
+            C acc = C(0);
+#pragma unroll
+            for (int r = 0; r <= PD; ++r) acc = fma(w[r], win[r], acc);
+            out[jr] = acc;
+            jr = jr + 1 == N ? 0 : jr + 1;
+#pragma unroll
+            for (int r = 0; r < PD; ++r) win[r] = win[r + 1];
+        }
+        return;
+    }
+    const double *xe = sgeo + PD;  // xe[c] = t_c, c in [-PD, N+PD]
+    const double *xi = sgeo + N + 2 * PD + 1;
+    const int *tbl = reinterpret_cast<const int *>(xi + N);  // bucket -> cell of its left edge
+    const int MT = P.adv_nbkt;
+    const double x0 = xe[0], xN = xe[N], Lp = xN - x0, invLp = 1.0 / Lp, bscale = MT * invLp;
+    constexpr int U = PD <= 3 ? 4 : 2;
+    for (int j0 = lane; j0 < N; j0 += 32 * U) {
+        double X[U];
+        int lo[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int jr = min(j0 + 32 * u, N - 1);
+            double x = xi[jr] - sh;
+            x -= floor((x - x0) * invLp) * Lp;
+            if (x < x0) x += Lp;
+            if (x >= xN) x -= Lp;
+            if (!(x >= x0 && x < xN)) x = x0;
+            int g = tbl[min(max((int)((x - x0) * bscale), 0), MT - 1)];
+            while (g + 1 < N && xe[g + 1] <= x) ++g;  // t_g <= x < t_{g+1}
+            while (g > 0 && xe[g] > x) --g;
+            X[u] = x;
+            lo[u] = g;
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            double dl[PD], dr[PD], b[PD + 1];
+#pragma unroll
+            for (int j = 0; j < PD; ++j) {
+                dl[j] = X[u] - xe[lo[u] - j];
+                dr[j] = xe[lo[u] + 1 + j] - X[u];
+            }
+            bspl_values<PD>(dl, dr, b);
+            int idx = lo[u] - PD + s;
+            idx = idx < 0 ? idx + N : idx;
+            C acc = C(0);
+#pragma unroll
+            for (int r = 0; r <= PD; ++r) {
+                acc = fma((C)b[r], coef[idx], acc);
+                idx = idx + 1 == N ? 0 : idx + 1;
+            }
+            if (j0 + 32 * u < N) out[j0 + 32 * u] = acc;
+        }
+    }
+}
+
+template <typename T, int K, int L, bool BULK, bool ADV>
 __global__ void __launch_bounds__(256)
     sb_warp_kernel(const __grid_constant__ KParams p) {
     using C = T;
@@ -664,6 +790,12 @@ __global__ void __launch_bounds__(256)
         fence_mbar_init();
     }
     stage_constants<C, K>(p, G, smem, tid, blockDim.x);
+    double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);  // advect, non-uniform: xe[N+2p+1] | xi[n] | bucket table
+    if (ADV && !P.adv_uniform) {
+        copy_words(sgeo, P.xe, P.N + 2 * P.p + 1, tid, blockDim.x);
+        copy_words(sgeo + P.N + 2 * P.p + 1, P.xi, n, tid, blockDim.x);
+        copy_words(reinterpret_cast<int *>(sgeo + P.N + 2 * P.p + 1 + n), P.adv_tbl, P.adv_nbkt, tid, blockDim.x);
+    }
     __syncthreads();
 
     const C *sL = reinterpret_cast<const C *>(smem + p.off_L);
@@ -682,7 +814,8 @@ __global__ void __launch_bounds__(256)
     const C *sdscale = reinterpret_cast<const C *>(smem + p.off_dscale);
     const int *sdrow = reinterpret_cast<const int *>(smem + p.off_drow);
     // per warp: row buffer(s) of n values + k spare for x1
-    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * (BULK ? 2 : 1) * p.wbuf_pitch;
+    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * ((BULK ? 2 : 1) + (ADV ? 1 : 0)) * p.wbuf_pitch;
+    C *outrow = wbuf + (size_t)(BULK ? 2 : 1) * p.wbuf_pitch;  // ADV: the advected row
 
     const int s = lane;
     const bool active = s < S;
@@ -796,14 +929,28 @@ __global__ void __launch_bounds__(256)
 #pragma unroll
         for (int i = 0; i < L; ++i)
             if (active && a + i < nQ) rowbuf[s_lo + a + i] = v[i][0];
+        C *res = rowbuf;  // row that goes back to HBM
+        if (ADV) {
+            // ---------- Algorithm 2: f(xi_i) <- S(xi_i - shift) while the coefficients are on chip
+            __syncwarp();
+            const double sh = p.shift[rhs];
+            switch (P.p) {  // degrees 1..5 (the library's range)
+                case 1: advect_row<C, 1>(P, sgeo, rowbuf, outrow, sh, lane); break;
+                case 2: advect_row<C, 2>(P, sgeo, rowbuf, outrow, sh, lane); break;
+                case 3: advect_row<C, 3>(P, sgeo, rowbuf, outrow, sh, lane); break;
+                case 4: advect_row<C, 4>(P, sgeo, rowbuf, outrow, sh, lane); break;
+                default: advect_row<C, 5>(P, sgeo, rowbuf, outrow, sh, lane); break;
+            }
+            res = outrow;
+        }
         if (BULK) {
             fence_proxy_async_smem();  // generic smem writes -> visible to the bulk copy
             __syncwarp();
             if (lane == 0) {
-                bulk_store(g, rowbuf, row_bytes);
+                bulk_store(g, res, row_bytes);
                 const int64_t nr = rhs + 2 * nw;  // next row for this buffer
+                if (ADV || nr < p.batch) bulk_wait_read();  // the store has read its source row
                 if (nr < p.batch) {
-                    bulk_wait_read();  // the store has read the buffer
                     mbar_arrive_expect_tx(wbar + (j & 1), row_bytes);
                     bulk_load(rowbuf, gout + nr * p.bstride, row_bytes, wbar + (j & 1));
                 }
@@ -812,12 +959,12 @@ __global__ void __launch_bounds__(256)
         } else if (vec) {
             __syncwarp();
             V *gv = reinterpret_cast<V *>(g);
-            const V *sv = reinterpret_cast<const V *>(rowbuf);
+            const V *sv = reinterpret_cast<const V *>(res);
             for (int q = lane; q < n / VW; q += 32) __stcs(gv + q, sv[q]);
             __syncwarp();
         } else {
             __syncwarp();
-            for (int q = lane; q < n; q += 32) __stcs(g + (int64_t)q * ps, (T)rowbuf[q]);
+            for (int q = lane; q < n; q += 32) __stcs(g + (int64_t)q * ps, (T)res[q]);
             __syncwarp();
         }
     }
@@ -935,7 +1082,8 @@ int tile_K(int K, const KParams &kp, const CUtensorMap *tm, int grid, int thread
 
 template <typename T, int K, int L>
 int launch_warp1(const KParams &kp, int grid, cudaStream_t st, char *err, int errlen) {
-    auto fn = kp.bulk ? sb_warp_kernel<T, K, L, true> : sb_warp_kernel<T, K, L, false>;
+    auto fn = kp.adv ? (kp.bulk ? sb_warp_kernel<T, K, L, true, true> : sb_warp_kernel<T, K, L, false, true>)
+                     : (kp.bulk ? sb_warp_kernel<T, K, L, true, false> : sb_warp_kernel<T, K, L, false, false>);
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total) != cudaSuccess)
         return check_launch("cudaFuncSetAttribute(warp)", err, errlen);
     fn<<<grid, kp.warp_threads, kp.smem_total, st>>>(kp);

@@ -26,6 +26,7 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0) {
+    const size_t geo_bytes = (kp.adv && !P.adv_uniform) ? (size_t)(P.N + 2 * P.p + 1 + P.n) * 8 + (size_t)P.adv_nbkt * 4 : 0;
     size_t o = 0;
     auto take = [&](size_t bytes, size_t al) {
         o = align_up(o, al);
@@ -55,6 +56,7 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_dscale = take((size_t)k * esz, 16);
     kp.off_drow = take((size_t)k * 4, 16);
     kp.off_cbuf = take((size_t)4 * cbox * R * esz, 128);
+    kp.off_geo = take(geo_bytes, 16);
     kp.off_mbar = take((2 * NBOXMAX + 4) * 8, 8);
     kp.smem_total = (int)align_up(o, 16);
     return kp.smem_total;
@@ -63,6 +65,10 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
 int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem, char *err, int errlen) {
     const size_t esz = a.dtype == 0 ? 8 : 4;
     const DevSeg &G = P.seg[2];
+    if (G.S == 0 && a.shift) {
+        snprintf(err, errlen, "advect: n=%d too large for the warp kernel", P.n);
+        return 5;
+    }
     if (G.S == 0) {  // Q too long for 32 register segments: serial fallback
         KParams kp{};
         kp.P = P;
@@ -80,6 +86,8 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
     kp.bstride = a.bstride;
     kp.pstride = a.pstride;
     kp.wbuf_pitch = (int)align_up((size_t)P.n + P.k + 2, 4);
+    kp.shift = a.shift;
+    kp.adv = a.shift != nullptr;
     // bulk-copy pipeline when every row is one contiguous, 16-B aligned run;
     // fewer warps per block (or no second buffer) when shared memory is short
     const bool can_bulk = a.pstride == 1 && (a.bstride * (int64_t)esz) % 16 == 0 && (uintptr_t)a.rhs % 16 == 0 &&
@@ -91,8 +99,12 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         if (cfg < 3 && !can_bulk) continue;
         kp.bulk = bulk;
         kp.warp_threads = 32 * wpb;
-        layout_smem(kp, P, G, 1, esz, (size_t)wpb * (bulk ? 2 : 1) * kp.wbuf_pitch * esz);
+        layout_smem(kp, P, G, 1, esz, (size_t)wpb * ((bulk ? 2 : 1) + (kp.adv ? 1 : 0)) * kp.wbuf_pitch * esz);
         fits = kp.smem_total <= max_smem;
+    }
+    if (!fits && kp.adv) {
+        snprintf(err, errlen, "advect: n=%d needs more shared memory than a block has", P.n);
+        return 5;
     }
     if (!fits) {  // factors + one row do not fit: serial fallback
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
@@ -116,8 +128,8 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
     int max_smem = 0;
     cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
 
-    // point-contiguous / general strided layouts: warp-per-RHS kernel
-    if (a.bstride != 1) return launch_warp(P, a, num_sms, max_smem, err, errlen);
+    // point-contiguous / general strided layouts and the advection step: warp-per-RHS kernel
+    if (a.bstride != 1 || a.shift) return launch_warp(P, a, num_sms, max_smem, err, errlen);
 
     const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
     const int L = G.L;

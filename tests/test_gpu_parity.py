@@ -229,3 +229,61 @@ def test_large_n_paths(torch_cuda, n_points, bc, p, layout):
     got = t.cpu().numpy()
     got = got if layout == "batch" else got.T
     assert rel_coef_error(got, ref) <= TOL64
+
+
+@pytest.mark.parametrize("p,kind", [(1, "uniform"), (2, "uniform"), (3, "uniform"), (4, "uniform"), (5, "uniform"),
+                                    (3, "sin"), (4, "sin"), (5, "sin"), (3, "jitter"), (5, "jitter"),
+                                    (2, "sin"), (3, "uniform_array")])
+@pytest.mark.parametrize("layout", ["point", "batch"])
+def test_advect_step_parity(torch_cuda, p, kind, layout):
+    """NEXT f1: one Algorithm-2 advection step (spline build + evaluation at
+    the feet of the characteristics) fused in the warp kernel,
+    against the oracle's solve + evaluation."""
+    torch = torch_cuda
+    N = 1024 if kind == "uniform" else 1000
+    sb, o = make(p, N, PERIODIC, kind)
+    B = 300
+    f = inputs.rhs(sb.n, B, seed=31)
+    v = np.linspace(-4.0, 4.0, B)
+    shift = 0.37 * v / N * 3.0  # up to ~4.4 cells
+    ref = o.advect(f, shift)
+    sh = torch.from_numpy(shift).cuda()
+    t = torch.from_numpy(f if layout == "batch" else np.ascontiguousarray(f.T)).cuda()
+    sb.advect_(t, sh)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    got = got if layout == "batch" else got.T
+    assert rel_coef_error(got, ref) <= TOL64
+
+
+def test_advect_fp32_and_errors(torch_cuda):
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, SplineBuilderError
+    sb, o = make(3, 1024, PERIODIC, "uniform")
+    f = inputs.rhs(sb.n, 64, seed=32)
+    shift = np.linspace(-0.01, 0.01, 64)
+    ref = o.advect(f.astype(np.float32).astype(np.float64), shift)
+    t = torch.from_numpy(np.ascontiguousarray(f.T.astype(np.float32))).cuda()
+    sb.advect_(t, torch.from_numpy(shift).cuda())
+    torch.cuda.synchronize()
+    assert rel_coef_error(t.cpu().numpy().T.astype(np.float64), ref) <= TOL32
+    g = SplineBuilder(5, 1000, GREVILLE)
+    with pytest.raises(SplineBuilderError):
+        g.advect_(torch.zeros(1000, 4, dtype=torch.float64, device="cuda"),
+                  torch.zeros(4, dtype=torch.float64, device="cuda"))
+
+
+@pytest.mark.parametrize("kind", ["uniform", "sin"])
+def test_advect_shifts_beyond_period(torch_cuda, kind):
+    """Feet more than one period away (|shift| up to 5.3 domain lengths) and
+    exact cell multiples wrap like the oracle's periodic evaluation."""
+    torch = torch_cuda
+    sb, o = make(3, 512, PERIODIC, kind)
+    B = 96
+    f = inputs.rhs(sb.n, B, seed=33)
+    shift = np.concatenate([np.linspace(-5.3, 5.3, B - 32), np.arange(-16, 16) / 512.0])
+    ref = o.advect(f, shift)
+    t = torch.from_numpy(np.ascontiguousarray(f.T)).cuda()
+    sb.advect_(t, torch.from_numpy(shift).cuda())
+    torch.cuda.synchronize()
+    assert rel_coef_error(t.cpu().numpy().T, ref) <= TOL64
