@@ -56,6 +56,7 @@ def _load():
         lib.oracle_handle_solve.argtypes = [vp, dp, i64, i64, i64, i32]
         lib.oracle_eval.argtypes = [vp, dp, i32, dp, i64, dp]
         lib.oracle_advect.argtypes = [vp, dp, i64, i64, i64, dp, i32]
+        lib.oracle_solve_2d.argtypes = [vp, vp, dp, i64, i64, i32]
         _lib = lib
     return _lib
 
@@ -155,6 +156,27 @@ class Oracle:
         den = np.abs(s * b2).max(axis=0)
         den[den == 0] = 1.0
         return float((r / den).max())
+
+
+def solve_2d(o1: Oracle, o2: Oracle, f: np.ndarray, nthreads: int = 0) -> np.ndarray:
+    """Tensor-product coefficients: f of shape (batch, n2, n1)
+    or (n2, n1), dim 1 (o1) fastest; returns C = A1^{-1} F A2^{-T} per grid."""
+    c = np.array(f, dtype=np.float64, order="C", copy=True)
+    g = c.reshape((1,) + c.shape) if c.ndim == 2 else c
+    assert g.ndim == 3 and g.shape[1] == o2.n and g.shape[2] == o1.n
+    st = _lib.oracle_solve_2d(o1._h, o2._h, _ptr(g), int(g.shape[0]), int(o1.n * o2.n), int(nthreads))
+    if st:
+        raise RuntimeError(f"oracle solve_2d failed: {st}")
+    return c
+
+
+def eval_2d(o1: Oracle, o2: Oracle, coef: np.ndarray, xs: np.ndarray, ys: np.ndarray) -> np.ndarray:
+    """S(x, y) = sum_{j1,j2} C[j2][j1] B1_{j1}(x) B2_{j2}(y) on the grid xs x ys
+    (result [len(ys)][len(xs)]), by 1-D evaluations along each dimension."""
+    coef = np.asarray(coef, dtype=np.float64)
+    # along dim 2 first: G[y][j1] = sum_{j2} C[j2][j1] B2_{j2}(y)
+    G = np.stack([o2.eval(np.ascontiguousarray(coef[:, j1]), ys) for j1 in range(o1.n)], axis=1)
+    return np.stack([o1.eval(np.ascontiguousarray(G[q]), xs) for q in range(len(ys))], axis=0)
 
 
 def rel_coef_error(x: np.ndarray, ref: np.ndarray) -> float:

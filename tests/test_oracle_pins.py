@@ -412,3 +412,90 @@ def test_advect_smooth_profile_is_accurate():
     f = np.sin(2 * np.pi * xs)[:, None]
     out = o.advect(f, np.array([0.2345]))
     assert np.abs(out[:, 0] - np.sin(2 * np.pi * (xs - 0.2345))).max() < 1e-6
+
+
+# ------------------------------------------------- 2-D tensor product
+# Pins of oracle.solve_2d (NEXT row f3): the 2-D interpolation system
+# sum C[j2][j1] B1_j1(xi1) B2_j2(xi2) = F, written out as one big matrix from
+# scipy-built 1-D collocation matrices, a 2-D FFT closed form, scipy's own
+# per-axis interpolation, and tensor-product polynomial reproduction.
+
+def test_2d_kronecker_brute_force_scipy_matrices():
+    """vec(C) = (A2 (x) A1)^{-1} vec(F) with A1, A2 built by scipy (not the oracle)."""
+    x1 = mesh(7, "jitter")
+    x2 = mesh(5, "sin")
+    A1, _ = scipy_periodic_matrix(x1, 3)
+    A2, _, _ = scipy_clamped_matrix(x2, 4, GREVILLE)
+    o1, o2 = Oracle(3, 7, PERIODIC, x1), Oracle(4, 5 + 4, GREVILLE, x2)
+    F = rng(5).uniform(-1, 1, size=(3, o2.n, o1.n))
+    C = oracle.solve_2d(o1, o2, F)
+    big = np.kron(A2, A1)
+    for b in range(3):
+        ref = np.linalg.solve(big, F[b].reshape(-1)).reshape(o2.n, o1.n)
+        assert np.abs(C[b] - ref).max() <= 1e-12 * np.abs(ref).max()
+
+
+@pytest.mark.parametrize("p1,p2", [(3, 3), (4, 5), (5, 3)])
+def test_2d_uniform_periodic_fft_closed_form(p1, p2):
+    """Uniform periodic x uniform periodic: A1, A2 circulant, so A1 C A2^T = F is
+    a 2-D cyclic convolution: C = ifft2(fft2(F) / (fft(c2)[:, None] fft(c1)[None, :]))."""
+    n1, n2 = 24, 20
+    F = rng(6).uniform(-1, 1, size=(n2, n1))
+    c1, c2 = circulant_first_col(p1, n1), circulant_first_col(p2, n2)
+    ref = np.real(np.fft.ifft2(np.fft.fft2(F) / (np.fft.fft(c2)[:, None] * np.fft.fft(c1)[None, :])))
+    C = oracle.solve_2d(Oracle(p1, n1, PERIODIC), Oracle(p2, n2, PERIODIC), F)
+    assert np.abs(C - ref).max() <= 1e-13 * np.abs(ref).max()
+
+
+def test_2d_matches_scipy_per_axis_interpolation():
+    """Greville x Greville: scipy make_interp_spline along axis 1 then axis 0
+    (scipy's own batched-over-the-other-axis solves) gives the same coefficients."""
+    p1, p2, N1, N2 = 3, 5, 9, 11
+    x1, x2 = mesh(N1, "sin"), mesh(N2, "jitter")
+    t1, t2 = clamped_knots(x1, p1), clamped_knots(x2, p2)
+    g1, g2 = greville(t1, p1, N1 + p1), greville(t2, p2, N2 + p2)
+    g1[-1], g2[-1] = x1[-1], x2[-1]
+    F = rng(7).uniform(-1, 1, size=(N2 + p2, N1 + p1))
+    s1 = si.make_interp_spline(g1, F, k=p1, t=t1, axis=1)
+    s1c = np.moveaxis(s1.c, 0, 1)  # scipy keeps the interpolation axis first
+    s2 = si.make_interp_spline(g2, s1c, k=p2, t=t2, axis=0)
+    C = oracle.solve_2d(Oracle(p1, N1 + p1, GREVILLE, x1), Oracle(p2, N2 + p2, GREVILLE, x2), F)
+    assert np.abs(C - s2.c).max() <= 1e-12 * np.abs(C).max()
+
+
+@pytest.mark.parametrize("bc1,bc2", [(GREVILLE, HERMITE), (HERMITE, GREVILLE)])
+def test_2d_tensor_polynomial_reproduction(bc1, bc2):
+    """Data from P(x, y) = sum a_ab x^a y^b, a <= p1, b <= p2: the tensor spline
+    equals P everywhere (Hermite rows take the polynomial's derivatives)."""
+    p1, p2, N1, N2 = 3, 5, 8, 6
+    x1, x2 = mesh(N1, "jitter"), mesh(N2, "sin")
+    npts1 = N1 + p1 if bc1 == GREVILLE else N1 + 1
+    npts2 = N2 + p2 if bc2 == GREVILLE else N2 + 1
+    o1, o2 = Oracle(p1, npts1, bc1, x1), Oracle(p2, npts2, bc2, x2)
+    a = rng(8).uniform(-1, 1, size=(p1 + 1, p2 + 1))
+    P1 = [np.polynomial.Polynomial(np.eye(p1 + 1)[i]) for i in range(p1 + 1)]
+    P2 = [np.polynomial.Polynomial(np.eye(p2 + 1)[i]) for i in range(p2 + 1)]
+    r1, _, d1 = o1.rows()
+    r2, _, d2 = o2.rows()
+    F = np.zeros((o2.n, o1.n))
+    for ia in range(p1 + 1):
+        u = np.array([P1[ia].deriv(d)(x) if d else P1[ia](x) for x, d in zip(r1, d1)])
+        for ib in range(p2 + 1):
+            v = np.array([P2[ib].deriv(d)(y) if d else P2[ib](y) for y, d in zip(r2, d2)])
+            F += a[ia, ib] * np.outer(v, u)
+    C = oracle.solve_2d(o1, o2, F)
+    xs = rng(9).uniform(x1[0], x1[-1], size=7)
+    ys = rng(10).uniform(x2[0], x2[-1], size=5)
+    S = oracle.eval_2d(o1, o2, C, xs, ys)
+    ref = sum(a[ia, ib] * np.outer(P2[ib](ys), P1[ia](xs)) for ia in range(p1 + 1) for ib in range(p2 + 1))
+    assert np.abs(S - ref).max() <= 1e-12 * max(1.0, np.abs(ref).max())
+
+
+def test_2d_interpolation_property_periodic_nonuniform():
+    """S(xi1_i1, xi2_i2) = F[i2][i1] on a non-uniform periodic x periodic grid."""
+    o1 = Oracle(4, 12, PERIODIC, mesh(12, "jitter"))
+    o2 = Oracle(3, 10, PERIODIC, mesh(10, "sin"))
+    F = rng(11).uniform(-1, 1, size=(o2.n, o1.n))
+    C = oracle.solve_2d(o1, o2, F)
+    S = oracle.eval_2d(o1, o2, C, o1.rows()[0], o2.rows()[0])
+    assert np.abs(S - F).max() <= 1e-12
