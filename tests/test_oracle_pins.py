@@ -499,3 +499,49 @@ def test_2d_interpolation_property_periodic_nonuniform():
     C = oracle.solve_2d(o1, o2, F)
     S = oracle.eval_2d(o1, o2, C, o1.rows()[0], o2.rows()[0])
     assert np.abs(S - F).max() <= 1e-12
+
+
+# ------------------------------------- mixed boundary conditions (NEXT row f4)
+# bc = lo | (hi << 4): Hermite derivative rows at one end, Greville abscissae
+# elsewhere (the nbc abscissae next to a Hermite end are dropped; R13).
+
+def mixed_case(p, N, lo, hi, kind):
+    nbc = (p - 1) // 2 if p % 2 else p // 2
+    x = mesh(N, kind)
+    n_hermite = (lo == HERMITE) + (hi == HERMITE)
+    o = Oracle(p, N + p - nbc * n_hermite, lo | (hi << 4), x)
+    t = clamped_knots(x, p)
+    n = N + p
+    g = greville(t, p, n)
+    g[-1] = x[-1]
+    keep = [j for j in range(n) if not ((lo == HERMITE and 1 <= j <= nbc) or (hi == HERMITE and n - 1 - nbc <= j <= n - 2))]
+    return o, x, t, g[keep], nbc
+
+
+@pytest.mark.parametrize("p", [2, 3, 4, 5])
+@pytest.mark.parametrize("lo,hi", [(HERMITE, GREVILLE), (GREVILLE, HERMITE)])
+@pytest.mark.parametrize("kind", ["uniform", "jitter"])
+def test_mixed_bc_matches_scipy(p, lo, hi, kind):
+    """scipy make_interp_spline on the clamped knots with the derivative
+    conditions on one side only (bc_type=(derivs, None) / (None, derivs))."""
+    o, x, t, pts, nbc = mixed_case(p, 20, lo, hi, kind)
+    g = rng(12)
+    y = g.uniform(-1, 1, len(pts))
+    dv = g.uniform(-1, 1, nbc)
+    conds = [(d + 1, dv[d]) for d in range(nbc)]
+    spl = si.make_interp_spline(pts, y, k=p, t=t, bc_type=(conds, None) if lo == HERMITE else (None, conds))
+    b = np.concatenate([dv, y]) if lo == HERMITE else np.concatenate([y, dv])
+    c = o.solve(b)
+    assert np.abs(c - spl.c).max() <= 1e-12 * max(1.0, np.abs(spl.c).max())
+
+
+@pytest.mark.parametrize("p", [3, 4, 5])
+@pytest.mark.parametrize("lo,hi", [(HERMITE, GREVILLE), (GREVILLE, HERMITE)])
+def test_mixed_bc_polynomial_reproduction(p, lo, hi):
+    o, x, t, pts, nbc = mixed_case(p, 17, lo, hi, "sin")
+    poly = np.polynomial.Polynomial(rng(13).uniform(-1, 1, p + 1))
+    xr, _, dr = o.rows()
+    b = np.array([poly.deriv(d)(xx) if d else poly(xx) for xx, d in zip(xr, dr)])
+    c = o.solve(b)
+    xs = rng(14).uniform(x[0], x[-1], 50)
+    assert np.abs(o.eval(c, xs) - poly(xs)).max() <= 1e-12
