@@ -38,6 +38,18 @@ METRIC = "RHS/s and achieved HBM GB/s (% of peak), cubic n=1000, 1e5 RHS, fp64"
 ADV_METRIC = "advection GLUPS (Eq. 7: Nx*Nv / step time), one Algorithm-2 step"
 STRONG = {"C5"}            # total batch fixed, sharded over the ranks
 ADVECT = {"ADV", "ADVNU"}  # one semi-Lagrangian step (Algorithm 2) per step, metric GLUPS (Eq. 7)
+SLAB_W = 2048  # C4M: RHS per slab (the v*mu extent)
+TWOD = {
+    # name: ((degree, n_points, bc, mesh) along dim 1, same along dim 2, grids per GPU, dtype, description)
+    "C6": ((3, 1024, 0, "uniform"), (3, 1024, 0, "uniform"), 64, "f64",
+           "C6 2-D tensor-product build (P:59): 64 grids of 1024 x 1024, cubic uniform periodic x periodic, fp64"),
+    "C6NU": ((3, 1024, 0, "sin"), (5, 1000, 1, "sin"), 64, "f64",
+             "C6 2-D tensor-product build: 64 grids, dim 1 cubic non-uniform periodic n=1024 x dim 2 quintic "
+             "non-uniform Greville n=1000, fp64"),
+    "C6F32": ((3, 1024, 0, "uniform"), (3, 1024, 0, "uniform"), 64, "f32",
+              "C6 2-D tensor-product build: 64 grids of 1024 x 1024, cubic uniform periodic, fp32"),
+}
+TWOD_METRIC = "2-D tensor-product build: grid points per second (n1*n2*grids / step time)"
 DEVICE_INPUT_ELEMS = 4e8   # above this, inputs are generated on the device (inputs.rhs_device)
 E2E_MAX_RHS = 1_000_000    # the e2e leg moves at most this many RHS through host memory
 
@@ -56,6 +68,9 @@ WORKLOADS = {
             "Algorithm 2 advection step: Nx=1024, Nv=1e5, cubic uniform periodic, x contiguous, fp64 (GLUPS)"),
     "ADVNU": (3, 1024, 0, "sin", 100000, "f64", "point",
               "Algorithm 2 advection step: Nx=1024, Nv=1e5, cubic non-uniform (sin map) periodic, fp64 (GLUPS)"),
+    "C4M": (3, 1024, 0, "uniform", 131072, "f64", "slabs",
+            "C4 second layout f[y=64][x=1024][v*mu=2048] cubic periodic along x (x in the middle: 64 slabs of "
+            "(1024, 2048) batch-contiguous blocks, spline_builder_solve_slabs), fp64"),
     "C5": (3, 1000, 0, "uniform", 8000000, "f64", "batch",
            "C5 cubic uniform periodic n=1000, 8e6 RHS in total sharded over the GPUs (strong scaling) fp64"),
 }
@@ -149,6 +164,8 @@ def make_rhs(deg, n, bc, B, first, layout, dtype):
     b = inputs.rhs(n, B, seed=1234, degree=deg, bc=bc, first=first)  # (n, B) fp64
     if layout == "point":
         b = np.ascontiguousarray(b.T)
+    elif layout == "slabs":  # f[y][x][v]: slab y = r // SLAB_W, column r % SLAB_W
+        b = np.ascontiguousarray(b.reshape(n, B // SLAB_W, SLAB_W).transpose(1, 0, 2))
     return np.ascontiguousarray(b.astype(np.float32 if dtype == "f32" else np.float64))
 
 
@@ -187,6 +204,162 @@ def cpu_oracle_rate(deg, npts, bc, knots, n, target_s=10.0, max_rhs=None, adv=Fa
     dt = time.perf_counter() - t0
     what = "solve + evaluation at the feet (Algorithm 2)" if adv else "dense GEPP oracle"
     return m / dt, threads, f"{m} RHS of the same workload (n={n}), {what}, {threads} OpenMP threads"
+
+
+def run_2d(args):
+    """2-D tensor-product workloads (NEXT row f3): a step = spline_builder_solve_2d
+    over every grid of this rank.  Algorithmic bytes = one read + one write of
+    every grid point (the single-pass minimum; two passes without L2 reuse
+    would move twice that)."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, solve_2d_
+
+    spec1, spec2, G, dt, desc = TWOD[args.workload]
+    ws, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    sbs = []
+    for deg, npts, bc, mesh in (spec1, spec2):
+        sbs.append(SplineBuilder(deg, npts, bc, inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh)))
+    n1, n2 = sbs[0].n, sbs[1].n
+    esz = 4 if dt == "f32" else 8
+    tdt = torch.float32 if dt == "f32" else torch.float64
+    host = inputs.rhs(n1, G * n2, seed=1234, first=rank * G * n2).T.reshape(G, n2, n1)
+    host = np.ascontiguousarray(host.astype(np.float32 if dt == "f32" else np.float64))
+    pristine = torch.from_numpy(host).cuda()
+    x = pristine.clone()
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    chunk_mb = int(os.environ.get("SB_2D_CHUNK_MB", "0"))
+    per_chunk = G if chunk_mb <= 0 else max(1, (chunk_mb << 20) // (n1 * n2 * esz))
+    launches_per_step = 2 * ((G + per_chunk - 1) // per_chunk)
+    CHUNK = 20
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    for _ in range(args.warmup):
+        solve_2d_(sbs[0], sbs[1], x)
+    barrier()
+    nchunks = (args.steps + CHUNK - 1) // CHUNK
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(nchunks)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(nchunks)]
+    with ClockSampler(local) as clk:
+        barrier()
+        done = 0
+        for c in range(nchunks):
+            m = min(CHUNK, args.steps - done)
+            x.copy_(pristine)
+            flush.fill_(c & 0xFF)
+            starts[c].record(stream)
+            for _ in range(m):
+                solve_2d_(sbs[0], sbs[1], x)
+            ends[c].record(stream)
+            done += m
+        barrier()
+    total_ms = float(sum(s_.elapsed_time(e_) for s_, e_ in zip(starts, ends)))
+    t_tensor = torch.tensor([total_ms], device="cuda", dtype=torch.float64)
+    if ws > 1:
+        dist.all_reduce(t_tensor, op=dist.ReduceOp.MAX)
+    ms_per_step = float(t_tensor[0]) / args.steps
+    pts = n1 * n2 * G
+    value = ws * pts / (ms_per_step / 1e3)
+    alg_bytes = 2.0 * pts * esz
+    achieved = alg_bytes / (ms_per_step / 1e3) / 1e9
+    peak, peak_kind = load_peaks()
+    e2e = None
+    if not args.no_e2e:
+        hp = torch.from_numpy(host.copy()).pin_memory()
+        dev = torch.empty_like(pristine)
+        ts = []
+        for _ in range(args.e2e_steps + 1):
+            barrier()
+            t0 = time.perf_counter()
+            dev.copy_(hp, non_blocking=True)
+            solve_2d_(sbs[0], sbs[1], dev)
+            hp.copy_(dev, non_blocking=True)
+            torch.cuda.synchronize()
+            ts.append(time.perf_counter() - t0)
+        te = torch.tensor([float(np.mean(ts[1:]))], device="cuda", dtype=torch.float64)
+        if ws > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": ws * pts / float(te[0]), "unit": "points/s", "h2d_bytes_per_step": int(host.nbytes),
+               "d2h_bytes_per_step": int(host.nbytes), "path": "H2D + spline_builder_solve_2d + D2H"}
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        import oracle
+        o1 = oracle.Oracle(spec1[0], spec1[1], spec1[2], inputs.breakpoints(inputs.n_cells(*spec1[:3]), spec1[3]))
+        o2 = oracle.Oracle(spec2[0], spec2[1], spec2[2], inputs.breakpoints(inputs.n_cells(*spec2[:3]), spec2[3]))
+        threads = len(os.sched_getaffinity(0))
+        t0 = time.perf_counter()
+        oracle.solve_2d(o1, o2, host[:1].astype(np.float64), nthreads=threads)
+        dt1 = time.perf_counter() - t0
+        m = int(max(1, min(G, 10.0 / max(dt1, 1e-6))))
+        t0 = time.perf_counter()
+        oracle.solve_2d(o1, o2, host[:m].astype(np.float64), nthreads=threads)
+        rate = m * n1 * n2 / (time.perf_counter() - t0)
+        cpu = {"value": rate, "unit": "points/s", "cores": threads, "kind": "oracle",
+               "sample": f"{m} of the {G} grids ({n1} x {n2}), dense GEPP oracle per dimension, {threads} threads"}
+    if rank == 0:
+        line = {
+            "metric": TWOD_METRIC, "value": value, "unit": "points/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": dt, "data": "synthetic (Philox U(-1,1) grids, seeded)",
+            "config": {"workload": desc, "n1": n1, "n2": n2, "grids_per_gpu": G, "l2_chunk_mb": chunk_mb,
+                       "l2": f"inputs {pts * esz / 1e6:.0f} MB per GPU > 126 MB L2; input restored + 256 MB L2 "
+                             f"flush every {CHUNK} steps (untimed)", "parallelism": f"dp{ws} (grid shards)"},
+            "achieved_gbs": achieved,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                         "traffic": None, "peak_kind": peak_kind, "kernel_ms": ms_per_step,
+                         "algorithmic_bytes_per_launch": alg_bytes / launches_per_step,
+                         "note": f"whole step ({launches_per_step} launches): one read + one write per point"},
+            "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches_per_step * args.steps, "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+def run_reference_2d(args):
+    """Reference arm of the 2-D workloads: the oracle's solve_2d as it stands on
+    a bounded sample of grids per step."""
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    spec1, spec2, G, dt, desc = TWOD[args.workload]
+    os_ = [oracle.Oracle(d, p, b, inputs.breakpoints(inputs.n_cells(d, p, b), m)) for d, p, b, m in (spec1, spec2)]
+    n1, n2 = os_[0].n, os_[1].n
+    threads = len(os.sched_getaffinity(0))
+    g0 = inputs.rhs(n1, n2, seed=1234).T.reshape(1, n2, n1).copy()
+    t0 = time.perf_counter()
+    oracle.solve_2d(os_[0], os_[1], g0, nthreads=threads)
+    dt1 = time.perf_counter() - t0
+    per_step = int(max(1, min(G, 100.0 / max(1, args.steps + args.warmup) / max(dt1, 1e-6))))
+    grids = inputs.rhs(n1, per_step * n2, seed=1234).T.reshape(per_step, n2, n1).copy()
+    for _ in range(args.warmup):
+        oracle.solve_2d(os_[0], os_[1], grids, nthreads=threads)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.solve_2d(os_[0], os_[1], grids, nthreads=threads)
+        times.append(time.perf_counter() - t0)
+    t = float(np.mean(times))
+    val = per_step * n1 * n2 / t
+    line = {
+        "impl": "reference", "metric": TWOD_METRIC, "value": val, "unit": "points/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": dt, "data": "synthetic",
+        "config": {"workload": desc, "n1": n1, "n2": n2, "grids_per_step": per_step},
+        "cpu_baseline": {"value": val, "unit": "points/s", "cores": threads, "kind": "oracle",
+                         "sample": f"{per_step} of the {G} grids per step"},
+        "e2e": {"value": val, "unit": "points/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
 
 
 def run_reference(args, wl):
@@ -242,12 +415,16 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS) + sorted(TWOD))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     args = ap.parse_args()
+    if args.workload in TWOD:
+        if args.impl == "reference":
+            return run_reference_2d(args)
+        return run_2d(args)
     wl = WORKLOADS[args.workload]
     if args.impl == "reference":
         return run_reference(args, wl)
@@ -287,6 +464,8 @@ def main():
     if adv:
         shift = torch.from_numpy(adv_shift(inputs.n_cells(deg, npts, bc), B, first)).cuda()
         step = lambda t: sb.advect_(t, shift)  # noqa: E731
+    elif layout == "slabs":
+        step = lambda t: sb.solve_slabs_(t, SLAB_W, SLAB_W, B // SLAB_W, n * SLAB_W)  # noqa: E731
     else:
         step = sb.solve_
 
@@ -387,7 +566,8 @@ def main():
             "vs_baseline": None, "dtype": dt, "data": "synthetic (Philox U(-1,1) RHS, seeded)",
             "config": {"workload": desc, "n": n, "batch_per_gpu": B, "batch_total": B_total, "degree": deg,
                        "bc": ["periodic", "greville", "hermite"][bc],
-                       "mesh": mesh, "layout": "batch-contiguous" if layout == "batch" else "point-contiguous",
+                       "mesh": mesh, "layout": {"batch": "batch-contiguous", "point": "point-contiguous",
+                                                "slabs": "slabs of batch-contiguous blocks"}[layout],
                        "l2": f"inputs {n * B * esz / 1e6:.0f} MB per GPU > 126 MB L2; input restored + 256 MB "
                              f"L2 flush every 40 steps (untimed)",
                        "inputs": "device Philox (inputs.rhs_device)" if on_device else "host Philox (inputs.rhs)",

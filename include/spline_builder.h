@@ -32,6 +32,8 @@ typedef struct spline_builder *spline_builder_t; /* opaque, immutable after crea
 
 /* boundary conditions (PAPER.md P:55 periodic; non-periodic per BASELINE C3) */
 enum { SB_PERIODIC = 0, SB_GREVILLE = 1, SB_HERMITE = 2 };
+/* different conditions at the two ends (Greville / Hermite only; R13) */
+#define SB_BC(lo, hi) ((lo) == (hi) ? (lo) : ((lo) | ((hi) << 4)))
 /* element types of the right-hand sides */
 enum { SB_F64 = 0, SB_F32 = 1 };
 /* status codes */
@@ -60,7 +62,12 @@ enum {
  *                       Greville  N = n_points - p      (n = N + p)
  *                       Hermite   N = n_points - 1 (odd p) or N = n_points
  *                                 (even p, values at cell midpoints); n = N + p
- *   bc       SB_PERIODIC, SB_GREVILLE or SB_HERMITE (both ends alike).
+ *   bc       SB_PERIODIC, SB_GREVILLE or SB_HERMITE (both ends alike), or
+ *            SB_BC(lo, hi) with lo != hi in {SB_GREVILLE, SB_HERMITE}: mixed,
+ *            N = n_points - p + nbc(lo) + nbc(hi), nbc(Hermite end) = nbc
+ *            below, nbc(Greville end) = 0; the value rows are the Greville
+ *            abscissae of the clamped basis without the nbc next to a Hermite
+ *            end (the end point itself stays).
  *   knots    NULL -> uniform mesh on [0, 1] (all cells of width 1/N exactly);
  *            else N+1 strictly increasing breakpoints (host pointer, read
  *            during the call only; the periodic period is knots[N]-knots[0]).
@@ -72,6 +79,8 @@ enum {
  *   Hermite: [f^(1..nbc)(x_0), f(x_0) ... f(x_N), f^(1..nbc)(x_N)] with raw
  *     derivatives (odd p, nbc = (p-1)/2); even p: values at the N cell
  *     midpoints, nbc = p/2.
+ *   mixed: [f^(1..nbc)(x_0) if lo is Hermite, values at the kept Greville
+ *     abscissae in increasing order, f^(1..nbc)(x_N) if hi is Hermite].
  * The handle owns host and device copies of the factors on the CUDA device
  * current at the call.  Returns NULL on failure (see last_error / the
  * status in spline_builder_last_status()).
@@ -112,6 +121,41 @@ int spline_builder_solve_f32(spline_builder_t h, float *rhs, int64_t batch, int6
  * in elements, > 0, and the (j, r) -> offset map must be one-to-one. */
 int spline_builder_solve_strided(spline_builder_t h, void *rhs, int dtype, int64_t batch, int64_t batch_stride,
                                  int64_t point_stride, void *stream);
+
+/*
+ * spline_builder_solve_slabs -- in-place solve of nslab independent
+ * batch-contiguous (n, batch) blocks in ONE launch: element (row j, rhs r,
+ * slab q) at rhs[q*slab_stride + j*ld + r].  This is the layout of a
+ * dimension that is neither the fastest nor the slowest of a higher-
+ * dimensional array (e.g. f[y][x][v] solved along x, slabs y), and pass 2 of
+ * the tensor-product builder below.  PAPER.md P:59: "batched over the other
+ * dimensions".
+ *   rhs          DEVICE pointer, SB_F64 or SB_F32 (dtype), caller owned.
+ *   ld >= batch  elements between rows;  slab_stride: elements between slabs,
+ *                either >= n*ld (stacked slabs) or >= batch with
+ *                ld >= (nslab-1)*slab_stride + batch (slabs side by side in
+ *                each row); anything that aliases -> SB_INVALID_ARG.
+ * nslab == 0 or batch == 0 is a no-op.  Asynchronous on stream.
+ */
+int spline_builder_solve_slabs(spline_builder_t h, void *rhs, int dtype, int64_t batch, int64_t ld, int64_t nslab,
+                               int64_t slab_stride, void *stream);
+
+/*
+ * spline_builder_solve_2d -- tensor-product spline coefficients (PAPER.md
+ * "Higher dimensional B-splines can be obtained by a tensor product of
+ * 1D splines.  For N-D splines, N equations in the form of equation (2) must
+ * be solved ... batched over the other dimensions"):  for each of the batch
+ * 2-D grids F (n2 x n1, dim 1 contiguous), in place
+ *     C = A1^{-1} F A2^{-T},   i.e. vec(C) = (A2 (x) A1)^{-1} vec(F),
+ * A1 / A2 the collocation matrices of h1 (along dim 1) and h2 (along dim 2).
+ * Element (i1, i2, b) at rhs[b*batch_stride + i2*n1 + i1], n1 = nbasis(h1),
+ * n2 = nbasis(h2); batch_stride >= n1*n2 (ignored when batch == 1).
+ * Two fused 1-D passes: dim 1 by the warp-per-RHS kernel (rows contiguous),
+ * dim 2 by the tile kernel over slabs (3-D TMA).  Both handles on the same
+ * device.  Asynchronous on stream.
+ */
+int spline_builder_solve_2d(spline_builder_t h1, spline_builder_t h2, void *rhs, int dtype, int64_t batch,
+                            int64_t batch_stride, void *stream);
 
 /*
  * spline_builder_advect -- one step of the 1-D semi-Lagrangian advection of

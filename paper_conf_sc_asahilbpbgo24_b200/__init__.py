@@ -17,7 +17,12 @@ from ._lib import (SB_F32, SB_F64, SB_FLAG_HOST_ONLY, SB_GREVILLE, SB_HERMITE, S
 
 PERIODIC, GREVILLE, HERMITE = SB_PERIODIC, SB_GREVILLE, SB_HERMITE
 
-__all__ = ["SplineBuilder", "SplineBuilderError", "PERIODIC", "GREVILLE", "HERMITE", "load_library"]
+
+def bc_mixed(lo: int, hi: int) -> int:
+    """SB_BC(lo, hi) of include/spline_builder.h: different conditions at x_0 / x_N."""
+    return lo if lo == hi else lo | (hi << 4)
+
+__all__ = ["SplineBuilder", "SplineBuilderError", "PERIODIC", "GREVILLE", "HERMITE", "load_library", "solve_2d_", "bc_mixed"]
 
 
 def load_library():
@@ -129,6 +134,18 @@ class SplineBuilder:
                                                           _stream_handle(stream)))
         return rhs
 
+    def solve_slabs_(self, rhs, batch: int, ld: int, nslab: int, slab_stride: int, stream=None):
+        """In-place solve of nslab batch-contiguous (n, batch) blocks, element
+        (j, r, q) at rhs[q*slab_stride + j*ld + r] (spline_builder_solve_slabs)."""
+        import torch
+        if not rhs.is_cuda:
+            raise ValueError("rhs must be a CUDA tensor")
+        dt = SB_F64 if rhs.dtype == torch.float64 else SB_F32
+        _lib.check(self._lib.spline_builder_solve_slabs(self._h, ctypes.c_void_p(rhs.data_ptr()), dt, int(batch),
+                                                        int(ld), int(nslab), int(slab_stride),
+                                                        _stream_handle(stream)))
+        return rhs
+
     def advect_(self, f, shift, batch_stride: int | None = None, stream=None):
         """One semi-Lagrangian step of Algorithm 2, in
         place: every RHS line of f (CUDA tensor, layouts as :meth:`solve_`) is
@@ -186,3 +203,23 @@ class SplineBuilder:
         _lib.check(self._lib.spline_builder_solve_cpu_plan(self._h, ctypes.c_void_p(arr.ctypes.data),
                                                            int(arr.shape[1]), 1, int(arr.shape[1])))
         return arr
+
+
+def solve_2d_(h1: SplineBuilder, h2: SplineBuilder, f, stream=None):
+    """Tensor-product coefficients in place (spline_builder_solve_2d):
+    f is a contiguous CUDA tensor of shape (batch, n2, n1) or (n2, n1), dim 1
+    (h1, size n1) fastest; on exit C = A1^{-1} F A2^{-T} for every grid."""
+    import torch
+    if not f.is_cuda or not f.is_contiguous():
+        raise ValueError("f must be a contiguous CUDA tensor")
+    if f.dtype not in (torch.float64, torch.float32):
+        raise TypeError("f must be float64 or float32")
+    shp = tuple(f.shape)
+    if len(shp) == 2:
+        shp = (1,) + shp
+    if len(shp) != 3 or shp[1] != h2.n or shp[2] != h1.n:
+        raise ValueError(f"f must have shape (batch, {h2.n}, {h1.n})")
+    dt = SB_F64 if f.dtype == torch.float64 else SB_F32
+    _lib.check(h1._lib.spline_builder_solve_2d(h1._h, h2._h, ctypes.c_void_p(f.data_ptr()), dt, int(shp[0]),
+                                               int(shp[1] * shp[2]), _stream_handle(stream)))
+    return f

@@ -19,7 +19,7 @@ SB_FLAG_HOST_ONLY = 1
 # every symbol include/spline_builder.h declares (checked by tests/test_abi.py)
 EXPORTS = [
     "spline_builder_create", "spline_builder_create_ex", "spline_builder_solve", "spline_builder_solve_f32",
-    "spline_builder_solve_strided", "spline_builder_advect", "spline_builder_solve_host", "spline_builder_destroy",
+    "spline_builder_solve_strided", "spline_builder_solve_slabs", "spline_builder_solve_2d", "spline_builder_advect", "spline_builder_solve_host", "spline_builder_destroy",
     "spline_builder_get_info", "spline_builder_nbasis", "spline_builder_get_blocks",
     "spline_builder_solve_cpu_plan", "spline_builder_last_error", "spline_builder_last_status",
     "spline_builder_version",
@@ -64,6 +64,10 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         getattr(lib, name).argtypes = [vp, dp, i64, i64, vp]
     lib.spline_builder_solve_strided.restype = i32
     lib.spline_builder_solve_strided.argtypes = [vp, dp, i32, i64, i64, i64, vp]
+    lib.spline_builder_solve_slabs.restype = i32
+    lib.spline_builder_solve_slabs.argtypes = [vp, dp, i32, i64, i64, i64, i64, vp]
+    lib.spline_builder_solve_2d.restype = i32
+    lib.spline_builder_solve_2d.argtypes = [vp, vp, dp, i32, i64, i64, vp]
     lib.spline_builder_advect.restype = i32
     lib.spline_builder_advect.argtypes = [vp, dp, i32, i64, i64, i64, dp, vp]
     lib.spline_builder_solve_host.restype = i32

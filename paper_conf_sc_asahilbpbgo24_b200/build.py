@@ -26,6 +26,8 @@ SOURCES = [
     ("tile_f32.cu", "cu"),
     ("warp_f64.cu", "cu"),
     ("warp_f32.cu", "cu"),
+    ("warp_adv_f64.cu", "cu"),
+    ("warp_adv_f32.cu", "cu"),
     ("serial.cu", "cu"),
 ]
 HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh"]

@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -142,7 +143,7 @@ int upload(spline_builder *h) {
         rowf[(size_t)i * (2 * K + 1) + 2 * K] = P.dinv[i];
     }
     size_t oRowf[2] = {pk.addv(rowf), pk.addv(conv<float>(rowf))};
-    size_t oXe = pk.addv(P.xe), oXi = pk.addv(P.xi), oTbl = pk.addv(P.adv_tbl);
+    size_t oXe = pk.addv(P.xe), oXi = pk.addv(P.xi), oRcp = pk.addv(P.adv_rcp), oTbl = pk.addv(P.adv_tbl);
     size_t oLam[2], oGam[2], oDlu[2], oDs[2];
     for (int c = 0; c < 2; ++c) {
         auto put = [&](const std::vector<double> &v) { return c == 0 ? pk.addv(v) : pk.addv(conv<float>(v)); };
@@ -187,7 +188,9 @@ int upload(spline_builder *h) {
     }
     d.xe = (const double *)at(oXe); d.xi = (const double *)at(oXi);
     d.adv_uniform = P.adv_uniform ? 1 : 0; d.adv_invh = P.adv_invh; d.adv_q0 = P.adv_q0;
+    d.adv_rcp = (const double *)at(oRcp);
     d.adv_tbl = (const int *)at(oTbl); d.adv_nbkt = (int)P.adv_tbl.size();
+    d.adv_bscale = P.xe.empty() ? 0.0 : (double)P.adv_tbl.size() / (P.xb[P.N] - P.xb[0]);
     d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
     d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);
     d.dpiv = (const int *)at(o_dpiv); d.drow = (const int *)at(o_drow);
@@ -195,7 +198,7 @@ int upload(spline_builder *h) {
 }
 
 int do_solve(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t bstride, int64_t pstride,
-             cudaStream_t stream, const double *shift = nullptr) {
+             cudaStream_t stream, const double *shift = nullptr, int64_t nslab = 1, int64_t slab_stride = 0) {
     if (!h) return fail(SB_INVALID_ARG, "null handle");
     if (h->host_only) return fail(SB_UNSUPPORTED, "handle was created with SB_FLAG_HOST_ONLY");
     if (dtype != SB_F64 && dtype != SB_F32) return fail(SB_INVALID_ARG, "dtype must be SB_F64 or SB_F32");
@@ -211,11 +214,24 @@ int do_solve(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t bst
     int cur = -1;
     cudaGetDevice(&cur);
     if (cur != h->device) cudaSetDevice(h->device);
-    sb::SolveArgs a{rhs, batch, bstride, pstride, dtype, stream, shift};
+    sb::SolveArgs a{rhs, batch, bstride, pstride, dtype, stream, shift, nslab, slab_stride};
     char err[256] = {0};
     int st = sb::launch_solve(h->dp, a, h->num_sms, err, sizeof(err));
     if (cur != h->device) cudaSetDevice(cur);
     if (st) return fail(st, err);
+    return SB_OK;
+}
+
+// slabs interleaved inside each row: columns [s*slab_stride, s*slab_stride+batch)
+// of one (n, ld) batch-contiguous block; contiguous when slab_stride == batch
+int do_solve_cols(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t ld, int64_t nslab,
+                  int64_t slab_stride, cudaStream_t stream) {
+    if (slab_stride == batch) return do_solve(h, rhs, dtype, nslab * batch, 1, ld, stream);
+    const size_t esz = dtype == SB_F64 ? 8 : 4;
+    for (int64_t sl = 0; sl < nslab; ++sl) {
+        const int st = do_solve(h, (char *)rhs + (size_t)(sl * slab_stride) * esz, dtype, batch, 1, ld, stream);
+        if (st) return st;
+    }
     return SB_OK;
 }
 
@@ -273,6 +289,62 @@ int spline_builder_advect(spline_builder_t h, void *f, int dtype, int64_t batch,
     if (h->plan.bc != sb::PERIODIC) return fail(SB_UNSUPPORTED, "advect needs a periodic spline space");
     if (batch > 0 && !shift) return fail(SB_INVALID_ARG, "shift is NULL");
     return do_solve(h, f, dtype, batch, batch_stride, point_stride, (cudaStream_t)stream, shift);
+}
+
+int spline_builder_solve_slabs(spline_builder_t h, void *rhs, int dtype, int64_t batch, int64_t ld, int64_t nslab,
+                               int64_t slab_stride, void *stream) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (nslab < 0) return fail(SB_INVALID_ARG, "nslab < 0");
+    if (nslab == 0 || batch == 0) return SB_OK;
+    if (ld < batch) return fail(SB_INVALID_ARG, "need ld >= batch");
+    const int64_t n = h->plan.n;
+    // one-to-one: slabs stacked (slab_stride >= n*ld) or interleaved inside each row
+    const bool stacked = slab_stride >= n * ld;
+    const bool inrow = slab_stride >= batch && ld >= (nslab - 1) * slab_stride + batch;
+    if (nslab > 1 && !stacked && !inrow) return fail(SB_INVALID_ARG, "slabs alias: (row, rhs, slab) -> offset is not one-to-one");
+    if (nslab > 1 && inrow && !stacked)  // one batch-contiguous block of nslab*slab_stride columns
+        return do_solve_cols(h, rhs, dtype, batch, ld, nslab, slab_stride, (cudaStream_t)stream);
+    return do_solve(h, rhs, dtype, batch, 1, ld, (cudaStream_t)stream, nullptr, nslab, nslab > 1 ? slab_stride : 0);
+}
+
+int spline_builder_solve_2d(spline_builder_t h1, spline_builder_t h2, void *rhs, int dtype, int64_t batch,
+                            int64_t batch_stride, void *stream) {
+    if (!h1 || !h2) return fail(SB_INVALID_ARG, "null handle");
+    if (h1->host_only || h2->host_only) return fail(SB_UNSUPPORTED, "handle was created with SB_FLAG_HOST_ONLY");
+    if (h1->device != h2->device) return fail(SB_INVALID_ARG, "the two handles live on different devices");
+    if (dtype != SB_F64 && dtype != SB_F32) return fail(SB_INVALID_ARG, "dtype must be SB_F64 or SB_F32");
+    if (batch < 0) return fail(SB_INVALID_ARG, "batch < 0");
+    if (batch == 0) return SB_OK;
+    if (!rhs) return fail(SB_INVALID_ARG, "rhs is NULL");
+    const int64_t n1 = h1->plan.n, n2 = h2->plan.n, slice = n1 * n2;
+    if (batch > 1 && batch_stride < slice) return fail(SB_INVALID_ARG, "need batch_stride >= n1*n2");
+    if (batch == 1) batch_stride = slice;
+    const size_t esz = dtype == SB_F64 ? 8 : 4;
+    // Pass 1 (dim 1, contiguous rows) then pass 2 (dim 2, rows n1 apart).
+    // SB_2D_CHUNK_MB > 0 runs both passes chunk by chunk so a chunk is still in
+    // L2 when pass 2 reads it; measured on C6 (64 grids of 1024^2 fp64):
+    // unchunked 0.406 ms, 24 MB chunks 0.936, 96 MB 0.552 (launch tails), so the
+    // default is one chunk.
+    static const int64_t chunk_mb = [] {
+        const char *e = getenv("SB_2D_CHUNK_MB");
+        return e ? (int64_t)atoll(e) : (int64_t)0;  // measured: chunked launches lose more to tails than L2 saves
+    }();
+    int64_t cb = batch;
+    if (chunk_mb > 0) cb = std::max<int64_t>(1, (chunk_mb << 20) / (slice * (int64_t)esz));
+    cb = std::min(cb, batch);
+    for (int64_t b0 = 0; b0 < batch; b0 += cb) {
+        const int64_t nb = std::min(cb, batch - b0);
+        void *base = (char *)rhs + (size_t)(b0 * batch_stride) * esz;
+        int st;
+        if (batch_stride == slice)
+            st = do_solve(h1, base, dtype, nb * n2, n1, 1, (cudaStream_t)stream);
+        else
+            st = do_solve(h1, base, dtype, n2, n1, 1, (cudaStream_t)stream, nullptr, nb, batch_stride);
+        if (st) return st;
+        st = do_solve(h2, base, dtype, n1, 1, n1, (cudaStream_t)stream, nullptr, nb, batch_stride);
+        if (st) return st;
+    }
+    return SB_OK;
 }
 
 int spline_builder_solve_host(spline_builder_t h, void *host_rhs, int dtype, int64_t batch, int64_t ld) {

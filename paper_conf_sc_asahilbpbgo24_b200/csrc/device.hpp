@@ -35,8 +35,10 @@ struct DevPlan {
     const double *xe, *xi;   // periodic extended knots t_c at xe[c+p] (N+2p+1), n row positions
     int adv_uniform;         // uniform periodic mesh: Algorithm 2's evaluation is a per-row stencil
     double adv_invh, adv_q0; // 1/h, (xi_0 - x_0)/h
-    const int *adv_tbl;      // non-uniform: bucket b of [x_0, x_N) in adv_nbkt -> cell of its left edge
+    const double *adv_rcp;   // non-uniform: 1/(t_{m+w} - t_m) at [(m+p)*p + w-1], m in [-p, N+p), w = 1..p
+    const int *adv_tbl;      // non-uniform: bucket b of [x_0, x_N) -> cell of its left edge (bucket <= min cell)
     int adv_nbkt;
+    double adv_bscale;       // adv_nbkt / (x_N - x_0)
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
     DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),
                              // [2] warp-per-RHS kernel (odd L; S == 0 if unavailable)
@@ -50,6 +52,8 @@ struct SolveArgs {
     int dtype;         // 0 fp64, 1 fp32
     cudaStream_t stream;
     const double *shift = nullptr;  // advect: per-RHS displacement (device, fp64); nullptr = plain solve
+    int64_t nslab = 1;              // independent (n, batch) blocks, slab_stride elements apart
+    int64_t slab_stride = 0;
 };
 
 // returns 0 on success, else an SB_* status; fills err on failure

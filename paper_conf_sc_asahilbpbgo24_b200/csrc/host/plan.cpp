@@ -464,16 +464,37 @@ void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, 
 Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi) {
     P = Plan();
     if (degree < 1 || degree > 5) return {1, "degree must be in 1..5"};
-    if (bc != PERIODIC && bc != GREVILLE && bc != HERMITE) return {1, "unknown boundary condition"};
+    // bc < 16: both ends alike; else lo | (hi << 4) (mixed, R13)
+    int bc_lo = bc, bc_hi = bc;
+    if (bc >= 16) {
+        bc_lo = bc & 15;
+        bc_hi = (bc >> 4) & 15;
+        if ((bc >> 8) || bc_lo == PERIODIC || bc_hi == PERIODIC) return {1, "unknown boundary condition"};
+        if (bc_lo == bc_hi) bc = bc_lo;
+    }
+    if (bc_lo != PERIODIC && bc_lo != GREVILLE && bc_lo != HERMITE) return {1, "unknown boundary condition"};
+    if (bc_hi != PERIODIC && bc_hi != GREVILLE && bc_hi != HERMITE) return {1, "unknown boundary condition"};
+    const bool mixed = bc_lo != bc_hi;
     P.p = degree;
     P.bc = bc;
+    P.bc_lo = bc_lo;
+    P.bc_hi = bc_hi;
+    const int nbc_p = (degree % 2) ? (degree - 1) / 2 : degree / 2;
     if (bc == PERIODIC) { P.N = n_points; P.n = P.N; }
     else if (bc == GREVILLE) { P.N = n_points - degree; P.n = P.N + degree; }
-    else {
+    else if (!mixed) {
         P.N = (degree % 2) ? n_points - 1 : n_points;
-        P.nbc = (degree % 2) ? (degree - 1) / 2 : degree / 2;
+        P.nbc = nbc_p;
         P.n = P.N + degree;
+    } else {
+        P.nbc_lo = bc_lo == HERMITE ? nbc_p : 0;
+        P.nbc_hi = bc_hi == HERMITE ? nbc_p : 0;
+        P.nbc = std::max(P.nbc_lo, P.nbc_hi);
+        P.N = n_points - degree + P.nbc_lo + P.nbc_hi;
+        P.n = P.N + degree;
+        if (P.n < P.nbc_lo + P.nbc_hi + 2) return {1, "too few points for this degree / boundary condition"};
     }
+    if (!mixed) P.nbc_lo = P.nbc_hi = (bc == HERMITE) ? P.nbc : 0;
     if (P.N < 1) return {1, "too few points for this degree / boundary condition"};
     if (bc == PERIODIC && P.N < 2) return {1, "periodic spline needs at least 2 cells"};
     const int N = P.N, n = P.n, p = P.p;
@@ -482,11 +503,27 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         P.h[c] = knots ? knots[c + 1] - knots[c] : 1.0 / (double)N;  // uniform: exact equal widths (R1)
         if (!(P.h[c] > 0.0) || !std::isfinite(P.h[c])) return {1, "breakpoints must be strictly increasing"};
     }
-    Space S{p, bc, N, n, P.nbc, P.h.data()};
+    Space S{p, bc == PERIODIC ? PERIODIC : GREVILLE, N, n, P.nbc, P.h.data()};  // clamped knots unless periodic
     // rows
     std::vector<RowPt> rows(n);
     P.rowscale.assign(n, 1.0);
-    if (bc != HERMITE) {
+    if (mixed) {
+        // derivative rows at a Hermite end; the Greville abscissae minus the nbc
+        // next to a Hermite end (the end point itself stays)
+        int r = 0;
+        for (int d = 1; d <= P.nbc_lo; ++d) { rows[r] = RowPt{S.span_of_cell(0), 0.0, d}; P.rowscale[r] = std::pow(P.h[0], d); ++r; }
+        for (int j = 0; j < n; ++j) {
+            if (j >= 1 && j <= P.nbc_lo) continue;
+            if (j >= n - 1 - P.nbc_hi && j <= n - 2) continue;
+            rows[r++] = greville(S, j);
+        }
+        for (int d = 1; d <= P.nbc_hi; ++d) {
+            rows[r] = RowPt{S.span_of_cell(N - 1), P.h[N - 1], d};
+            P.rowscale[r] = std::pow(P.h[N - 1], d);
+            ++r;
+        }
+        if (r != n) return {1, "mixed boundary rows do not add up"};
+    } else if (bc != HERMITE) {
         for (int j = 0; j < n; ++j) rows[j] = greville(S, j);
     } else {
         int r = 0;
@@ -532,12 +569,26 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         P.adv_uniform = dev <= 2.3e-16 * xmax;
         P.adv_invh = 1.0 / hu;
         P.adv_q0 = (P.xi[0] - P.xb[0]) / hu;
-        P.adv_tbl.resize(2 * N);
-        for (int b = 0, c = 0; b < 2 * N; ++b) {
-            const double x = P.xb[0] + b * (Lp / (2.0 * N));
-            while (c + 1 < N && P.xb[c + 1] <= x) ++c;
-            P.adv_tbl[b] = c;
+        // bucket table: buckets no wider than the smallest cell, so the cell of a
+        // point is the bucket's cell or the next one
+        {
+            double hmin = Lp;
+            for (int c = 0; c < N; ++c) hmin = std::min(hmin, P.xb[c + 1] - P.xb[c]);
+            const int MT = (int)std::min<double>(8.0 * N, std::ceil(Lp / hmin * (1.0 + 1e-12)));
+            P.adv_tbl.resize(std::max(MT, 1));
+            for (int b = 0, c = 0; b < (int)P.adv_tbl.size(); ++b) {
+                const double x = P.xb[0] + b * (Lp / P.adv_tbl.size());
+                while (c + 1 < N && P.xb[c + 1] <= x) ++c;
+                P.adv_tbl[b] = c;
+            }
         }
+        // reciprocal knot differences 1/(t_{m+w} - t_m), m in [-p, N+p), w = 1..p:
+        // the denominators of de Boor's recursion depend on the knots only, so the
+        // non-uniform evaluation multiplies instead of dividing
+        P.adv_rcp.assign((size_t)(N + 2 * p) * p, 0.0);
+        for (int m = -p; m < N + p; ++m)
+            for (int w = 1; w <= p; ++w)
+                if (m + w <= N + p) P.adv_rcp[(size_t)(m + p) * p + (w - 1)] = 1.0 / (P.xe[m + w + p] - P.xe[m + p]);
     }
     // equilibrated sparse rows: rowscale * (d^deriv B_j)(point)
     P.A.assign(n, SparseRow());
@@ -569,11 +620,11 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         for (int k = std::max(kl, ku); k <= std::min(n, KMAX_DELTA); ++k) cands.push_back({0, k});
     } else {
         // score candidates by (kernel band K, kl+ku, k)
-        const int lo0 = (bc == HERMITE) ? P.nbc : 0;
+        const int lo0 = P.nbc_lo, hi0 = P.nbc_hi;  // derivative rows always go to delta
         struct C { int K, bw, k, a, b; };
         std::vector<C> cs;
         for (int a = lo0; a <= lo0 + p + 1; ++a)
-            for (int b = lo0; b <= lo0 + p + 1; ++b) {
+            for (int b = hi0; b <= hi0 + p + 1; ++b) {
                 if (a + b > KMAX_DELTA || a + b >= n) continue;
                 int kl = 0, ku = 0;
                 for (int i = a; i < n - b; ++i)

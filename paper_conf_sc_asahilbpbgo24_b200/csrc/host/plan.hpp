@@ -39,13 +39,15 @@ struct SegPlan {
 struct Plan {
     // ---- spline space
     int p = 0, bc = 0, N = 0, n = 0, nbc = 0;
+    int bc_lo = 0, bc_hi = 0, nbc_lo = 0, nbc_hi = 0;  // per end (mixed boundary conditions)
     std::vector<double> h;          // cell widths
     std::vector<double> xb;         // N+1 breakpoints (xb[N] = xb[0] + period for periodic)
     std::vector<double> xi;         // n interpolation points (row positions; derivative rows: the end point)
     std::vector<double> xe;         // periodic: extended knots t_c, c in [-p, N+p] at xe[c+p]
     bool adv_uniform = false;       // periodic uniform mesh (stencil evaluation of Algorithm 2)
     double adv_invh = 0.0, adv_q0 = 0.0;  // 1/h and (xi_0 - x_0)/h
-    std::vector<int> adv_tbl;       // 2N buckets of [x_0, x_N): cell containing the bucket's left edge
+    std::vector<int> adv_tbl;       // periodic: buckets of [x_0, x_N) no wider than the smallest cell -> cell
+    std::vector<double> adv_rcp;    // periodic: 1/(t_{m+w} - t_m) at [(m+p)*p + w-1], m in [-p, N+p), w = 1..p
     std::vector<SparseRow> A;       // equilibrated collocation matrix rows
     std::vector<double> rowscale;   // A_eq = diag(rowscale) * A_raw
     // ---- Schur split (Eq. 3)

@@ -44,6 +44,7 @@ namespace sb {
 
 enum Loader { LOAD_DIRECT = 0, LOAD_TMA = 1 };
 constexpr int NBOXMAX = 8;
+constexpr int WB_FRONT = 4;  // warp kernel: elements in front of each row buffer (advection wrap pad)
 constexpr int TILE_MAX_THREADS = 512;  // <= 15 compute warps + 1 corner/producer warp: 4 warps per
                                        // SM sub-partition keeps the 128-register budget
 
@@ -52,6 +53,8 @@ struct KParams {
     void *rhs;
     int64_t batch, bstride, pstride;
     int ntiles, nbox, boxr, ncw;     // tiles, TMA boxes per tile, rows per box, compute warps
+    int tps;                         // tile kernel: tiles per slab (ntiles = nslab * tps)
+    int64_t slab_stride;             // tile kernel: elements between slabs of (n, batch) blocks
     int empty_count[NBOXMAX];        // arrivals that free box c (reader warps; corner warp if none)
     int corner_arrive_mask;          // boxes without a compute-warp reader: the corner warp frees them
     int cbox;                        // rows of each corner box (0: corner reads the main tile)
@@ -62,7 +65,8 @@ struct KParams {
     int wbuf_pitch;                  // warp kernel: elements per per-warp row buffer
     int bulk, warp_threads;          // warp kernel: bulk-copy pipeline on/off, threads per block
     const double *shift;             // advect: per-RHS displacement (nullptr: plain solve)
-    int adv, off_geo;                // advect flag; smem offset of xb[N+1], hw[N], xi[n] (fp64)
+                                     // (wbuf_pitch includes WB_FRONT + n + max(k, 3) + slack)
+    int adv, off_geo;                // advect flag; smem offset of xe[N+2p+1], xi[n], rcp[(N+2p) p] (fp64)
 };
 
 // ------------------------------------------------------------- PTX helpers
@@ -95,6 +99,16 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, u
         "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
             smem_u32(dst)),
         "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(mbar))
+        : "memory");
+}
+// 3-D box (rhs, row, slab): the tile kernel's tensor maps carry a slab
+// dimension so one launch covers many (n, batch) blocks (2-D builder, pass 2)
+__device__ __forceinline__ void tma_load_3d(void *dst, const CUtensorMap *map, uint64_t *mbar, int c0, int c1,
+                                            int c2) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+        "[%5];" ::"r"(smem_u32(dst)),
+        "l"(map), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(mbar))
         : "memory");
 }
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
@@ -375,19 +389,22 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         const uint32_t cbytes = (uint32_t)(2 * cbox * R * sizeof(T));
         auto issue_cbox = [&](int t, int b) {
             T *dst = cbuf + (size_t)b * 2 * cbox * R;
+            const int sl = t / p.tps, tb = t - sl * p.tps;
             mbar_arrive_expect_tx(cfull + b, cbytes);
-            tma_load_2d(dst, &tmap_c, cfull + b, t * R, 0);
-            tma_load_2d(dst + (size_t)cbox * R, &tmap_c, cfull + b, t * R, P.n - cbox);
+            tma_load_3d(dst, &tmap_c, cfull + b, tb * R, 0, sl);
+            tma_load_3d(dst + (size_t)cbox * R, &tmap_c, cfull + b, tb * R, P.n - cbox, sl);
         };
         if (use_cbox && lane == 0 && (int)blockIdx.x < p.ntiles) issue_cbox(blockIdx.x, 0);
         int it = 0;
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
+            const int slab = tile / p.tps, tb = tile - slab * p.tps;
+            T *gs = gout + slab * p.slab_stride;
             if (LOADER == LOAD_TMA) {
                 if (lane == 0) {
                     for (int c = 0; c < nbox; ++c) {
                         if (it > 0) mbar_wait(empty + c, (it - 1) & 1);
                         mbar_arrive_expect_tx(full + c, box_bytes);
-                        tma_load_2d(buf + (size_t)c * boxr * R, &tmap, full + c, tile * R, c * boxr);
+                        tma_load_3d(buf + (size_t)c * boxr * R, &tmap, full + c, tb * R, c * boxr, slab);
                     }
                     if (use_cbox && tile + (int)gridDim.x < p.ntiles) issue_cbox(tile + gridDim.x, (it + 1) & 1);
                 }
@@ -398,9 +415,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 mbar_wait(empty + 0, (it - 1) & 1);  // all compute warps finished tile it-1
             }
             const T *cb = cbuf + (size_t)(it & 1) * 2 * cbox * R;
-            const int64_t ccol = (int64_t)tile * R + rr;
+            const int64_t ccol = (int64_t)tb * R + rr;
             const bool clive = ccol < p.batch;
-            const T *ccolp = gout + ccol * p.bstride;
+            const T *ccolp = gs + ccol * p.bstride;
             auto ldb = [&](int row) -> C {
                 if (LOADER == LOAD_TMA) {
                     if (use_cbox) return (C)cb[(size_t)(row < cbox ? row : cbox + row - (P.n - cbox)) * R + rr];
@@ -430,7 +447,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             if (part == 0 && k > 0) {
                 getrs_small(x1, sdlu, sdpiv, k);
                 if (clive)
-                    for (int d = 0; d < k; ++d) __stcs(gout + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
+                    for (int d = 0; d < k; ++d) __stcs(gs + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
             }
             __syncwarp();
             if (part == 0) mbar_arrive(x1full + (it & 1));
@@ -469,10 +486,11 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const int nthr_c = ncw * 32;
     int it = 0;
     for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
-        const int64_t col0 = (int64_t)tile * R + r0;
+        const int slab = tile / p.tps;
+        const int64_t col0 = (int64_t)(tile - slab * p.tps) * R + r0;
         // right-hand sides of this thread that exist (0..NV)
         const int nlive = active ? (int)max((int64_t)0, min((int64_t)NV, p.batch - col0)) : 0;
-        T *gcol = gout + col0 * p.bstride;
+        T *gcol = gout + slab * p.slab_stride + col0 * p.bstride;
         C v[L][NV];
         // ---------- own segment of b0 into registers
         if (LOADER == LOAD_TMA) {
@@ -670,104 +688,132 @@ __device__ __forceinline__ void bspl_values(const double (&dl)[PD], const double
     }
 }
 
+// Non-uniform periodic evaluation at a foot x in cell c (Algorithm 2's
+// interpolation step): de Boor's triangular recursion (BSPLVB) with the
+// denominators t_{c+1+r} - t_{c-j+r} replaced by precomputed reciprocals, so
+// no division; knots, reciprocals and the p+1 coefficients come straight from
+// shared memory through two base pointers (immediate offsets).  The
+// coefficients are coef[(c-p+s+r) mod N]; the row is padded on both sides
+// (coef[-2..-1] = coef[N-2..N-1], coef[N..N+2] = coef[0..2]), so no wrap.
+template <typename C, int PD>
+__device__ __forceinline__ C nu_value(double x, int c, const double *xe, const C *coef, const double *rc) {
+    constexpr int s = (PD + 1) / 2;
+    const double *tk = xe + c;       // tk[q] = t_{c+q}
+    const double *rk = rc + c * PD;  // rk[m*PD + w-1] = 1/(t_{c+m+w} - t_{c+m})
+    double b[PD + 1];
+    b[0] = 1.0;
+#pragma unroll
+    for (int j = 0; j < PD; ++j) {
+        double saved = 0.0;
+#pragma unroll
+        for (int r = 0; r <= j; ++r) {
+            const double term = b[r] * rk[(r - j) * PD + j];  // 1/(t_{c+1+r} - t_{c-j+r})
+            b[r] = fma(tk[1 + r] - x, term, saved);
+            saved = (x - tk[r - j]) * term;
+        }
+        b[j + 1] = saved;
+    }
+    const C *cw = coef + (c - PD + s);
+    C acc = C(0);
+#pragma unroll
+    for (int r = 0; r <= PD; ++r) acc = fma((C)b[r], cw[r], acc);
+    return acc;
+}
+
 // One row of the advection step.
 // Uniform mesh: every foot xi_i - shift has the same local coordinate u, so
 // the weights are computed once per row and out[i] = sum_r w_r coef[i+off+r]
 // is a (p+1)-tap stencil.  Lane l owns the run of window starts
 // [l*M, l*M+M) (M odd: conflict-free smem strides) and slides a register
 // window along it: ~N + 32p shared loads per row instead of (p+1) N.
-// Otherwise: per point, locate the cell through the bucket table, then
-// BSPLVB; U independent points per iteration for latency hiding.
 template <typename C, int PD>
-__device__ __forceinline__ void advect_row(const DevPlan &P, const double *sgeo, const C *coef, C *out, double sh,
-                                           int lane) {
+__device__ __forceinline__ void advect_row(const DevPlan &P, const C *coef, C *out, double sh, int lane) {
     constexpr int s = (PD + 1) / 2;
     const int N = P.N;
-    if (P.adv_uniform) {
-        const double q = P.adv_q0 - sh * P.adv_invh;  // foot of point 0, in cells from x_0
-        const double cf = floor(q);
-        double dl[PD], dr[PD], b[PD + 1];
+    const double q = P.adv_q0 - sh * P.adv_invh;  // foot of point 0, in cells from x_0
+    const double cf = floor(q);
+    double dl[PD], dr[PD], b[PD + 1];
 #pragma unroll
-        for (int j = 0; j < PD; ++j) {
-            dl[j] = (q - cf) + j;
-            dr[j] = (j + 1) - (q - cf);
-        }
-        bspl_values<PD>(dl, dr, b);
-        C w[PD + 1];
-#pragma unroll
-        for (int r = 0; r <= PD; ++r) w[r] = (C)b[r];
-        int c0 = (int)(cf - (double)N * floor(cf / (double)N));
-        c0 = c0 >= N ? c0 - N : (c0 < 0 ? c0 + N : c0);
-        int off = c0 - PD + s;  // point i reads coef[i + off .. i + off + PD] (mod N)
-        off = off < 0 ? off + N : (off >= N ? off - N : off);
-        const int M = ((N + 31) >> 5) | 1;
-        const int cbeg = lane * M;
-        if (cbeg >= N) return;
-        const int cend = min(cbeg + M, N);
-        C win[PD + 1];
-        int idx = cbeg;
-#pragma unroll
-        for (int r = 0; r < PD; ++r) {
-            win[r] = coef[idx];
-            idx = idx + 1 == N ? 0 : idx + 1;
-        }
-        int jr = cbeg - off;
-        jr = jr < 0 ? jr + N : jr;
-        for (int c = cbeg; c < cend; ++c) {
-            win[PD] = coef[idx];
-            idx = idx + 1 == N ? 0 : idx + 1;
-            C acc = C(0);
-#pragma unroll
-            for (int r = 0; r <= PD; ++r) acc = fma(w[r], win[r], acc);
-            out[jr] = acc;
-            jr = jr + 1 == N ? 0 : jr + 1;
-#pragma unroll
-            for (int r = 0; r < PD; ++r) win[r] = win[r + 1];
-        }
-        return;
+    for (int j = 0; j < PD; ++j) {
+        dl[j] = (q - cf) + j;
+        dr[j] = (j + 1) - (q - cf);
     }
-    const double *xe = sgeo + PD;  // xe[c] = t_c, c in [-PD, N+PD]
-    const double *xi = sgeo + N + 2 * PD + 1;
-    const int *tbl = reinterpret_cast<const int *>(xi + N);  // bucket -> cell of its left edge
+    bspl_values<PD>(dl, dr, b);
+    C w[PD + 1];
+#pragma unroll
+    for (int r = 0; r <= PD; ++r) w[r] = (C)b[r];
+    int c0 = (int)(cf - (double)N * floor(cf / (double)N));
+    c0 = c0 >= N ? c0 - N : (c0 < 0 ? c0 + N : c0);
+    int off = c0 - PD + s;  // point i reads coef[i + off .. i + off + PD] (mod N)
+    off = off < 0 ? off + N : (off >= N ? off - N : off);
+    const int M = ((N + 31) >> 5) | 1;
+    const int cbeg = lane * M;
+    if (cbeg >= N) return;
+    const int cend = min(cbeg + M, N);
+    C win[PD + 1];
+    int idx = cbeg;
+#pragma unroll
+    for (int r = 0; r < PD; ++r) {
+        win[r] = coef[idx];
+        idx = idx + 1 == N ? 0 : idx + 1;
+    }
+    int jr = cbeg - off;
+    jr = jr < 0 ? jr + N : jr;
+    for (int c = cbeg; c < cend; ++c) {
+        win[PD] = coef[idx];
+        idx = idx + 1 == N ? 0 : idx + 1;
+        C acc = C(0);
+#pragma unroll
+        for (int r = 0; r <= PD; ++r) acc = fma(w[r], win[r], acc);
+        out[jr] = acc;
+        jr = jr + 1 == N ? 0 : jr + 1;
+#pragma unroll
+        for (int r = 0; r < PD; ++r) win[r] = win[r + 1];
+    }
+}
+
+// Non-uniform mesh: lanes take consecutive points (j = lane + 32u, two per
+// iteration for ILP); the foot's cell comes from a bucket table (bucket width
+// <= the smallest cell, so at most one step to correct) and nu_value
+// evaluates the p+1 B-splines there.  Results go straight to HBM, coalesced
+// (the row is on chip, so the in-place write is safe): no output buffer.
+template <typename C, typename T, int PD>
+__device__ __forceinline__ void advect_row_nu(const DevPlan &P, const double *sgeo, const C *coef, T *g,
+                                              int64_t ps, double sh, int lane) {
+    const int N = P.N;
+    const double *xe = sgeo + PD;               // xe[c] = t_c, c in [-PD, N+PD]
+    const double *xi = sgeo + N + 2 * PD + 1;   // interpolation points (n = N)
+    const double *rc = xi + N + PD * PD;        // rc[m*PD + w-1] = 1/(t_{m+w} - t_m), m in [-PD, N+PD)
+    const int *tbl = reinterpret_cast<const int *>(rc + (N + PD) * PD);
     const int MT = P.adv_nbkt;
-    const double x0 = xe[0], xN = xe[N], Lp = xN - x0, invLp = 1.0 / Lp, bscale = MT * invLp;
-    constexpr int U = PD <= 3 ? 4 : 2;
-    for (int j0 = lane; j0 < N; j0 += 32 * U) {
-        double X[U];
-        int lo[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int jr = min(j0 + 32 * u, N - 1);
-            double x = xi[jr] - sh;
-            x -= floor((x - x0) * invLp) * Lp;
-            if (x < x0) x += Lp;
-            if (x >= xN) x -= Lp;
-            if (!(x >= x0 && x < xN)) x = x0;
-            int g = tbl[min(max((int)((x - x0) * bscale), 0), MT - 1)];
-            while (g + 1 < N && xe[g + 1] <= x) ++g;  // t_g <= x < t_{g+1}
-            while (g > 0 && xe[g] > x) --g;
-            X[u] = x;
-            lo[u] = g;
+    const double x0 = xe[0], xN = xe[N], Lp = xN - x0, invLp = 1.0 / Lp, bscale = P.adv_bscale;
+    double shr = sh - floor(sh * invLp) * Lp;  // sh mod L, in [0, L)
+    if (shr >= Lp) shr -= Lp;
+    if (shr < 0.0) shr += Lp;
+    auto locate = [&](double x) {  // t_c <= x < t_{c+1}
+        int c = tbl[min(max((int)((x - x0) * bscale), 0), MT - 1)];
+        c += (x >= xe[c + 1]);
+        if (x < xe[c] || x >= xe[c + 1]) {  // rounding at a bucket edge: walk
+            while (c > 0 && x < xe[c]) --c;
+            while (c + 1 < N && x >= xe[c + 1]) ++c;
         }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            double dl[PD], dr[PD], b[PD + 1];
-#pragma unroll
-            for (int j = 0; j < PD; ++j) {
-                dl[j] = X[u] - xe[lo[u] - j];
-                dr[j] = xe[lo[u] + 1 + j] - X[u];
-            }
-            bspl_values<PD>(dl, dr, b);
-            int idx = lo[u] - PD + s;
-            idx = idx < 0 ? idx + N : idx;
-            C acc = C(0);
-#pragma unroll
-            for (int r = 0; r <= PD; ++r) {
-                acc = fma((C)b[r], coef[idx], acc);
-                idx = idx + 1 == N ? 0 : idx + 1;
-            }
-            if (j0 + 32 * u < N) out[j0 + 32 * u] = acc;
-        }
+        return c;
+    };
+    auto foot = [&](int j) {
+        double x = xi[j] - shr;
+        if (x < x0) x += Lp;
+        if (x >= xN) x -= Lp;
+        return (x >= x0 && x < xN) ? x : x0;
+    };
+    for (int j0 = lane; j0 < N; j0 += 64) {
+        const int j1 = j0 + 32;
+        const bool v1 = j1 < N;
+        const double xa = foot(j0), xb = foot(v1 ? j1 : j0);
+        const int ca = locate(xa), cb = locate(xb);
+        const C ya = nu_value<C, PD>(xa, ca, xe, coef, rc);
+        const C yb = nu_value<C, PD>(xb, cb, xe, coef, rc);
+        __stcs(g + (int64_t)j0 * ps, (T)ya);
+        if (v1) __stcs(g + (int64_t)j1 * ps, (T)yb);
     }
 }
 
@@ -790,11 +836,14 @@ __global__ void __launch_bounds__(256)
         fence_mbar_init();
     }
     stage_constants<C, K>(p, G, smem, tid, blockDim.x);
-    double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);  // advect, non-uniform: xe[N+2p+1] | xi[n] | bucket table
+    // advect, non-uniform: xe[N+2p+1] | xi[n] | rcp[(N+2p) p] | bucket table (int)
+    double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);
     if (ADV && !P.adv_uniform) {
         copy_words(sgeo, P.xe, P.N + 2 * P.p + 1, tid, blockDim.x);
         copy_words(sgeo + P.N + 2 * P.p + 1, P.xi, n, tid, blockDim.x);
-        copy_words(reinterpret_cast<int *>(sgeo + P.N + 2 * P.p + 1 + n), P.adv_tbl, P.adv_nbkt, tid, blockDim.x);
+        copy_words(sgeo + P.N + 2 * P.p + 1 + n, P.adv_rcp, (P.N + 2 * P.p) * P.p, tid, blockDim.x);
+        copy_words(reinterpret_cast<int *>(sgeo + P.N + 2 * P.p + 1 + n + (P.N + 2 * P.p) * P.p), P.adv_tbl,
+                   P.adv_nbkt, tid, blockDim.x);
     }
     __syncthreads();
 
@@ -813,9 +862,11 @@ __global__ void __launch_bounds__(256)
     const int *sdpiv = reinterpret_cast<const int *>(smem + p.off_dpiv);
     const C *sdscale = reinterpret_cast<const C *>(smem + p.off_dscale);
     const int *sdrow = reinterpret_cast<const int *>(smem + p.off_drow);
-    // per warp: row buffer(s) of n values + k spare for x1
-    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * ((BULK ? 2 : 1) + (ADV ? 1 : 0)) * p.wbuf_pitch;
-    C *outrow = wbuf + (size_t)(BULK ? 2 : 1) * p.wbuf_pitch;  // ADV: the advected row
+    // per warp: row buffer(s) of WB_FRONT pad + n values + k spare for x1 (the
+    // advection pads the row on both sides); uniform advection: + an output row
+    const int nbuf = (BULK ? 2 : 1) + ((ADV && P.adv_uniform) ? 1 : 0);
+    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * nbuf * p.wbuf_pitch + WB_FRONT;
+    C *outrow = wbuf + (size_t)(BULK ? 2 : 1) * p.wbuf_pitch;  // ADV (uniform): the advected row
 
     const int s = lane;
     const bool active = s < S;
@@ -930,20 +981,50 @@ __global__ void __launch_bounds__(256)
         for (int i = 0; i < L; ++i)
             if (active && a + i < nQ) rowbuf[s_lo + a + i] = v[i][0];
         C *res = rowbuf;  // row that goes back to HBM
+        bool direct = false;  // the result was written to HBM by the evaluation itself
         if (ADV) {
             // ---------- Algorithm 2: f(xi_i) <- S(xi_i - shift) while the coefficients are on chip
-            __syncwarp();
             const double sh = p.shift[rhs];
-            switch (P.p) {  // degrees 1..5 (the library's range)
-                case 1: advect_row<C, 1>(P, sgeo, rowbuf, outrow, sh, lane); break;
-                case 2: advect_row<C, 2>(P, sgeo, rowbuf, outrow, sh, lane); break;
-                case 3: advect_row<C, 3>(P, sgeo, rowbuf, outrow, sh, lane); break;
-                case 4: advect_row<C, 4>(P, sgeo, rowbuf, outrow, sh, lane); break;
-                default: advect_row<C, 5>(P, sgeo, rowbuf, outrow, sh, lane); break;
+            if (P.adv_uniform) {
+                __syncwarp();
+                switch (P.p) {  // degrees 1..5 (the library's range)
+                    case 1: advect_row<C, 1>(P, rowbuf, outrow, sh, lane); break;
+                    case 2: advect_row<C, 2>(P, rowbuf, outrow, sh, lane); break;
+                    case 3: advect_row<C, 3>(P, rowbuf, outrow, sh, lane); break;
+                    case 4: advect_row<C, 4>(P, rowbuf, outrow, sh, lane); break;
+                    default: advect_row<C, 5>(P, rowbuf, outrow, sh, lane); break;
+                }
+                res = outrow;
+            } else {
+                // wrap pads: rowbuf[-2..-1] = rowbuf[n-2..n-1], rowbuf[n..n+2] = rowbuf[0..2]
+                __syncwarp();
+                if (lane < 2) rowbuf[lane - 2] = rowbuf[n - 2 + lane];
+                else if (lane < 5) rowbuf[n + lane - 2] = rowbuf[lane - 2];
+                __syncwarp();
+                switch (P.p) {
+                    case 1: advect_row_nu<C, T, 1>(P, sgeo, rowbuf, g, ps, sh, lane); break;
+                    case 2: advect_row_nu<C, T, 2>(P, sgeo, rowbuf, g, ps, sh, lane); break;
+                    case 3: advect_row_nu<C, T, 3>(P, sgeo, rowbuf, g, ps, sh, lane); break;
+                    case 4: advect_row_nu<C, T, 4>(P, sgeo, rowbuf, g, ps, sh, lane); break;
+                    default: advect_row_nu<C, T, 5>(P, sgeo, rowbuf, g, ps, sh, lane); break;
+                }
+                direct = true;
             }
-            res = outrow;
         }
-        if (BULK) {
+        if (BULK && direct) {
+            __syncwarp();  // every lane is done reading this row buffer
+            if (lane == 0) {
+                const int64_t nr = rhs + 2 * nw;
+                if (nr < p.batch) {
+                    fence_proxy_async_smem();  // generic reads before the async refill
+                    mbar_arrive_expect_tx(wbar + (j & 1), row_bytes);
+                    bulk_load(rowbuf, gout + nr * p.bstride, row_bytes, wbar + (j & 1));
+                }
+            }
+            __syncwarp();
+        } else if (direct) {
+            __syncwarp();
+        } else if (BULK) {
             fence_proxy_async_smem();  // generic smem writes -> visible to the bulk copy
             __syncwarp();
             if (lane == 0) {
@@ -1046,6 +1127,8 @@ int launch_tile_f32(int R, int loader, int K, const KParams &kp, const CUtensorM
                     cudaStream_t st, char *err, int errlen);
 int launch_warp_f64(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 int launch_warp_f32(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
+int launch_warp_adv_f64(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
+int launch_warp_adv_f32(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 int launch_serial(int dtype, int K, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 
 inline int check_launch(const char *what, char *err, int errlen) {
@@ -1080,10 +1163,9 @@ int tile_K(int K, const KParams &kp, const CUtensorMap *tm, int grid, int thread
     return 5;
 }
 
-template <typename T, int K, int L>
+template <typename T, int K, int L, bool ADV>
 int launch_warp1(const KParams &kp, int grid, cudaStream_t st, char *err, int errlen) {
-    auto fn = kp.adv ? (kp.bulk ? sb_warp_kernel<T, K, L, true, true> : sb_warp_kernel<T, K, L, false, true>)
-                     : (kp.bulk ? sb_warp_kernel<T, K, L, true, false> : sb_warp_kernel<T, K, L, false, false>);
+    auto fn = kp.bulk ? sb_warp_kernel<T, K, L, true, ADV> : sb_warp_kernel<T, K, L, false, ADV>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total) != cudaSuccess)
         return check_launch("cudaFuncSetAttribute(warp)", err, errlen);
     fn<<<grid, kp.warp_threads, kp.smem_total, st>>>(kp);
@@ -1091,27 +1173,30 @@ int launch_warp1(const KParams &kp, int grid, cudaStream_t st, char *err, int er
 }
 
 // odd segment lengths instantiated for the warp kernel (the plan picks from this set)
-template <typename T, int K>
+template <typename T, int K, bool ADV>
 int warp_L(int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen) {
     switch (L) {
-        case 3: return launch_warp1<T, K, 3>(kp, grid, st, err, errlen);
-        case 5: return launch_warp1<T, K, 5>(kp, grid, st, err, errlen);
-        case 9: return launch_warp1<T, K, 9>(kp, grid, st, err, errlen);
-        case 17: return launch_warp1<T, K, 17>(kp, grid, st, err, errlen);
-        case 33: return launch_warp1<T, K, 33>(kp, grid, st, err, errlen);
-        case 63: return launch_warp1<T, K, 63>(kp, grid, st, err, errlen);
+        case 3: return launch_warp1<T, K, 3, ADV>(kp, grid, st, err, errlen);
+        case 5: return launch_warp1<T, K, 5, ADV>(kp, grid, st, err, errlen);
+        case 9: return launch_warp1<T, K, 9, ADV>(kp, grid, st, err, errlen);
+        case 17: return launch_warp1<T, K, 17, ADV>(kp, grid, st, err, errlen);
+        case 33: return launch_warp1<T, K, 33, ADV>(kp, grid, st, err, errlen);
+        case 63: return launch_warp1<T, K, 63, ADV>(kp, grid, st, err, errlen);
     }
     snprintf(err, errlen, "warp kernel: no instantiation for segment length %d", L);
     return 5;
 }
 
-template <typename T>
+// ADV (the advection step) exists for periodic spaces only, whose Q band is <= 3
+template <typename T, bool ADV>
 int warp_K(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen) {
     switch (K) {
-        case 1: return warp_L<T, 1>(L, kp, grid, st, err, errlen);
-        case 2: return warp_L<T, 2>(L, kp, grid, st, err, errlen);
-        case 3: return warp_L<T, 3>(L, kp, grid, st, err, errlen);
-        case 4: return warp_L<T, 4>(L, kp, grid, st, err, errlen);
+        case 1: return warp_L<T, 1, ADV>(L, kp, grid, st, err, errlen);
+        case 2: return warp_L<T, 2, ADV>(L, kp, grid, st, err, errlen);
+        case 3: return warp_L<T, 3, ADV>(L, kp, grid, st, err, errlen);
+        case 4:
+            if constexpr (!ADV) return warp_L<T, 4, ADV>(L, kp, grid, st, err, errlen);
+            break;
     }
     snprintf(err, errlen, "unsupported band K=%d", K);
     return 5;

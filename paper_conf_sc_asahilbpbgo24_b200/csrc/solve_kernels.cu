@@ -26,7 +26,7 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0) {
-    const size_t geo_bytes = (kp.adv && !P.adv_uniform) ? (size_t)(P.N + 2 * P.p + 1 + P.n) * 8 + (size_t)P.adv_nbkt * 4 : 0;
+    const size_t geo_bytes = (kp.adv && !P.adv_uniform) ? (size_t)(P.N + 2 * P.p + 1 + P.n + (P.N + 2 * P.p) * P.p) * 8 + (size_t)P.adv_nbkt * 4 : 0;
     size_t o = 0;
     auto take = [&](size_t bytes, size_t al) {
         o = align_up(o, al);
@@ -85,22 +85,48 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
     kp.batch = a.batch;
     kp.bstride = a.bstride;
     kp.pstride = a.pstride;
-    kp.wbuf_pitch = (int)align_up((size_t)P.n + P.k + 2, 4);
+    kp.wbuf_pitch = (int)align_up((size_t)WB_FRONT + P.n + std::max(P.k, 3) + 2, 4);
     kp.shift = a.shift;
     kp.adv = a.shift != nullptr;
     // bulk-copy pipeline when every row is one contiguous, 16-B aligned run;
     // fewer warps per block (or no second buffer) when shared memory is short
     const bool can_bulk = a.pstride == 1 && (a.bstride * (int64_t)esz) % 16 == 0 && (uintptr_t)a.rhs % 16 == 0 &&
                           ((int64_t)P.n * (int64_t)esz) % 16 == 0;
-    bool fits = false;
-    for (int cfg = 0; cfg < 6 && !fits; ++cfg) {
-        const bool bulk = cfg < 3 && can_bulk;
-        const int wpb = (cfg % 3 == 0) ? (bulk ? 4 : 8) : (cfg % 3 == 1 ? 2 : 1);
-        if (cfg < 3 && !can_bulk) continue;
-        kp.bulk = bulk;
-        kp.warp_threads = 32 * wpb;
-        layout_smem(kp, P, G, 1, esz, (size_t)wpb * ((bulk ? 2 : 1) + (kp.adv ? 1 : 0)) * kp.wbuf_pitch * esz);
-        fits = kp.smem_total <= max_smem;
+    // candidates (bulk pipeline first, measured best for C4), scored by resident
+    // warps per SM; the per-block constants (factors, advection geometry) are
+    // paid once per block, so large-smem cases prefer fewer, wider blocks.
+    // SB_WARP_BULK=0/1 forces the loader (A/B experiments).
+    static const int bulk_env = [] {
+        const char *e = getenv("SB_WARP_BULK");
+        return e ? atoi(e) : -1;
+    }();
+    struct Cand { bool bulk; int wpb; };
+    const Cand cands[] = {{true, 4}, {true, 2}, {true, 1}, {true, 8}, {true, 6}, {true, 3},
+                          {false, 8}, {false, 6}, {false, 4}, {false, 2}, {false, 1}};
+    const int out_row = (kp.adv && P.adv_uniform) ? 1 : 0;  // uniform advection writes via an output row
+    int best = -1, best_score = 0;
+    for (int ci = 0; ci < (int)(sizeof(cands) / sizeof(cands[0])); ++ci) {
+        const Cand &c = cands[ci];
+        if (c.bulk && !can_bulk) continue;
+        if (bulk_env >= 0 && c.bulk != (bulk_env > 0)) continue;
+        KParams t = kp;
+        layout_smem(t, P, G, 1, esz, (size_t)c.wpb * ((c.bulk ? 2 : 1) + out_row) * kp.wbuf_pitch * esz);
+        if (t.smem_total > max_smem) continue;
+        const int per_sm = std::min(16 / c.wpb, (int)(228 * 1024 / (t.smem_total + 1024)));
+        // the bulk pipeline (double-buffered rows) is worth 1.5x the warps
+        // (measured: C4 bulk 12 warps/SM 0.378 ms vs plain 16 warps 0.396 ms)
+        const int score = c.wpb * std::max(per_sm, 1) * (c.bulk ? 3 : 2);
+        if (score > best_score) {
+            best_score = score;
+            best = ci;
+        }
+    }
+    const bool fits = best >= 0;
+    if (fits) {
+        kp.bulk = cands[best].bulk;
+        kp.warp_threads = 32 * cands[best].wpb;
+        layout_smem(kp, P, G, 1, esz,
+                    (size_t)cands[best].wpb * ((kp.bulk ? 2 : 1) + out_row) * kp.wbuf_pitch * esz);
     }
     if (!fits && kp.adv) {
         snprintf(err, errlen, "advect: n=%d needs more shared memory than a block has", P.n);
@@ -111,7 +137,7 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
     }
     const int wpb = kp.warp_threads / 32;
-    const int per_sm = std::max(1, std::min(8, (int)(228 * 1024 / (kp.smem_total + 1024))));
+    const int per_sm = std::max(1, std::min(16 / wpb, (int)(228 * 1024 / (kp.smem_total + 1024))));
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + wpb - 1) / wpb, (int64_t)num_sms * per_sm));
     // round L up to an instantiated odd length (the plan chose the smallest odd L >= nQ/32)
     if (a.dtype == 0) return launch_warp_f64(P.K, G.L, kp, grid, a.stream, err, errlen);
@@ -120,8 +146,21 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
 
 }  // namespace
 
-int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, int errlen) {
-    if (a.batch == 0) return 0;
+int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err, int errlen) {
+    SolveArgs a = a_in;
+    if (a.batch == 0 || a.nslab == 0) return 0;
+    if (a.nslab > 1 && (a.bstride != 1 || a.shift)) {
+        // slabs of a strided layout: the warp kernel takes them one launch each
+        for (int64_t sl = 0; sl < a.nslab; ++sl) {
+            SolveArgs b = a;
+            b.nslab = 1;
+            b.rhs = (char *)a.rhs + sl * a.slab_stride * (a.dtype == 0 ? 8 : 4);
+            const int st = launch_solve(P, b, num_sms, err, errlen);
+            if (st) return st;
+        }
+        return 0;
+    }
+    if (a.nslab == 1) a.slab_stride = (int64_t)P.n * a.pstride;
     const size_t esz = a.dtype == 0 ? 8 : 4;
     int dev = 0;
     cudaGetDevice(&dev);
@@ -130,6 +169,16 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
 
     // point-contiguous / general strided layouts and the advection step: warp-per-RHS kernel
     if (a.bstride != 1 || a.shift) return launch_warp(P, a, num_sms, max_smem, err, errlen);
+    auto per_slab_warp = [&]() {  // batch-contiguous slabs the tile kernel cannot take
+        for (int64_t sl = 0; sl < a.nslab; ++sl) {
+            SolveArgs b = a;
+            b.nslab = 1;
+            b.rhs = (char *)a.rhs + sl * a.slab_stride * (int64_t)esz;
+            const int st = launch_warp(P, b, num_sms, max_smem, err, errlen);
+            if (st) return st;
+        }
+        return 0;
+    };
 
     const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
     const int L = G.L;
@@ -139,8 +188,9 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
     kp.batch = a.batch;
     kp.bstride = a.bstride;
     kp.pstride = a.pstride;
-    // TMA needs a 16-B aligned base and row pitch; boxes of <= 256 rows
-    const bool aligned = ((uintptr_t)a.rhs % 16 == 0) && ((a.pstride * (int64_t)esz) % 16 == 0);
+    // TMA needs a 16-B aligned base, row pitch and slab pitch; boxes of <= 256 rows
+    const bool aligned = ((uintptr_t)a.rhs % 16 == 0) && ((a.pstride * (int64_t)esz) % 16 == 0) &&
+                         ((a.slab_stride * (int64_t)esz) % 16 == 0) && a.nslab < (1ll << 31);
     const int nbox = (P.n + 255) / 256;
     const int boxr = ((P.n + nbox - 1) / nbox + 7) / 8 * 8;
     const int cands64[2] = {16, 8}, cands32[2] = {32, 16};
@@ -160,11 +210,15 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
             loader = LOAD_DIRECT;
         }
     }
-    if (!R) return launch_warp(P, a, num_sms, max_smem, err, errlen);  // too large for the tile kernel
+    if (!R) return per_slab_warp();  // too large for the tile kernel
     const int RP = R / tile_nv((int)esz);  // a compute thread owns NV right-hand sides
     kp.ncw = (RP * G.S + 31) / 32;
     layout_smem(kp, P, G, R, esz, loader == LOAD_TMA ? (size_t)nbox * boxr * R * esz : 0);
-    kp.ntiles = (int)((a.batch + R - 1) / R);
+    const int64_t tps = (a.batch + R - 1) / R;
+    if (tps * a.nslab >= (1ll << 31)) return per_slab_warp();
+    kp.tps = (int)tps;
+    kp.ntiles = (int)(tps * a.nslab);
+    kp.slab_stride = a.slab_stride;
     kp.nbox = nbox;
     kp.boxr = boxr;
     // corner boxes: the corner reads only rows [0,cbox) and [n-cbox,n); they are
@@ -215,13 +269,13 @@ int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, i
     memset(tm, 0, sizeof(tm));
     if (loader == LOAD_TMA) {
         for (int q = 0; q < (cbox ? 2 : 1); ++q) {
-            cuuint64_t dims[2] = {(cuuint64_t)a.batch, (cuuint64_t)P.n};
-            cuuint64_t strides[1] = {(cuuint64_t)(a.pstride * (int64_t)esz)};
-            cuuint32_t box[2] = {(cuuint32_t)R, (cuuint32_t)(q == 0 ? boxr : cbox)};
-            cuuint32_t estr[2] = {1, 1};
+            cuuint64_t dims[3] = {(cuuint64_t)a.batch, (cuuint64_t)P.n, (cuuint64_t)a.nslab};
+            cuuint64_t strides[2] = {(cuuint64_t)(a.pstride * (int64_t)esz), (cuuint64_t)(a.slab_stride * (int64_t)esz)};
+            cuuint32_t box[3] = {(cuuint32_t)R, (cuuint32_t)(q == 0 ? boxr : cbox), 1};
+            cuuint32_t estr[3] = {1, 1, 1};
             CUresult cr = get_encode()(&tm[q], a.dtype == 0 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64
                                                             : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
-                                       2, a.rhs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                       3, a.rhs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             if (cr != CUDA_SUCCESS) {

@@ -24,9 +24,28 @@ PERIODIC, GREVILLE, HERMITE = 0, 1, 2
 RHS_BLOCK = 4096
 
 
+def bc_mixed(lo: int, hi: int) -> int:
+    """Boundary-condition code of include/spline_builder.h for (lo, hi) ends."""
+    return lo if lo == hi else lo | (hi << 4)
+
+
+def bc_ends(bc: int) -> tuple[int, int]:
+    return (bc, bc) if bc < 16 else (bc & 15, (bc >> 4) & 15)
+
+
+def n_hermite_rows(degree: int, bc: int) -> tuple[int, int]:
+    """Derivative rows at (x_0, x_N) -- the header's row-order convention."""
+    nbc = (degree - 1) // 2 if degree % 2 else degree // 2
+    lo, hi = bc_ends(bc)
+    return (nbc if lo == HERMITE else 0, nbc if hi == HERMITE else 0)
+
+
 def n_cells(degree: int, n_points: int, bc: int) -> int:
     """Number of cells N implied by (degree, n_points, bc) -- the counting
     convention of include/spline_builder.h, not method arithmetic."""
+    if bc >= 16:
+        lo, hi = n_hermite_rows(degree, bc)
+        return n_points - degree + lo + hi
     if bc == PERIODIC:
         return n_points
     if bc == GREVILLE:
@@ -75,11 +94,12 @@ def rhs(n: int, batch: int, seed: int = 1234, dtype=np.float64, degree: int = 3,
         lo, hi = max(first, q * RHS_BLOCK), min(first + batch, (q + 1) * RHS_BLOCK)
         b[lo - first:hi - first] = blk[lo - q * RHS_BLOCK:hi - q * RHS_BLOCK]
     b = b.T.copy()
-    if bc == HERMITE:
-        nbc = (degree - 1) // 2 if degree % 2 else degree // 2
-        for d in range(1, nbc + 1):
+    if bc != PERIODIC:
+        nlo, nhi = n_hermite_rows(degree, bc)
+        for d in range(1, nlo + 1):
             b[d - 1, :] *= (2.0 * np.pi) ** d
-            b[n - nbc + d - 1, :] *= (2.0 * np.pi) ** d
+        for d in range(1, nhi + 1):
+            b[n - nhi + d - 1, :] *= (2.0 * np.pi) ** d
     return np.ascontiguousarray(b.astype(dtype))
 
 

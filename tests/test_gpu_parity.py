@@ -60,6 +60,11 @@ CASES = [
     (5, 8, GREVILLE, "uniform"),
     (3, 33, PERIODIC, "uniform"),
     (3, 64, PERIODIC, "jitter"),
+    # mixed ends (NEXT row f4): Hermite at one end, Greville at the other
+    (5, 998, HERMITE | (GREVILLE << 4), "sin"),
+    (3, 200, GREVILLE | (HERMITE << 4), "jitter"),
+    (4, 150, HERMITE | (GREVILLE << 4), "uniform"),
+    (2, 60, GREVILLE | (HERMITE << 4), "sin"),
 ]
 
 
@@ -287,3 +292,128 @@ def test_advect_shifts_beyond_period(torch_cuda, kind):
     sb.advect_(t, torch.from_numpy(shift).cuda())
     torch.cuda.synchronize()
     assert rel_coef_error(t.cpu().numpy().T, ref) <= TOL64
+
+
+# ------------------------------------------- slabs (spline_builder_solve_slabs)
+@pytest.mark.parametrize("p,npts,bc,kind", [(3, 1000, PERIODIC, "uniform"), (5, 1000, GREVILLE, "sin"),
+                                            (5, 996, HERMITE, "sin"), (4, 200, PERIODIC, "jitter")])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_slabs_stacked_parity(torch_cuda, p, npts, bc, kind, dtype):
+    """nslab stacked (n, batch) blocks with padding (ld > batch, slab gap): one
+    launch of the tile kernel over a 3-D tensor map; each slab matches the oracle,
+    padding untouched."""
+    torch = torch_cuda
+    sb, orc = make(p, npts, bc, kind)
+    n, B, ld, nslab = sb.n, 37, 48, 5
+    sstride = n * ld + 16
+    buf = np.full(nslab * sstride, 7.0)
+    blocks = []
+    for q in range(nslab):
+        b = inputs.rhs(n, B, seed=50 + q, degree=p, bc=bc)
+        blocks.append(b)
+        for j in range(n):
+            buf[q * sstride + j * ld: q * sstride + j * ld + B] = b[j]
+    t = torch.from_numpy(buf.astype(dtype)).cuda()
+    sb.solve_slabs_(t, B, ld, nslab, sstride)
+    torch.cuda.synchronize()
+    out = t.cpu().numpy().astype(np.float64)
+    tol = TOL64 if dtype == np.float64 else TOL32
+    mask = np.ones_like(out, dtype=bool)
+    for q in range(nslab):
+        got = np.stack([out[q * sstride + j * ld: q * sstride + j * ld + B] for j in range(n)])
+        for j in range(n):
+            mask[q * sstride + j * ld: q * sstride + j * ld + B] = False
+        ref = orc.solve(blocks[q].astype(dtype).astype(np.float64))
+        assert rel_coef_error(got, ref) <= tol
+    assert np.all(out[mask] == 7.0)
+
+
+def test_slabs_side_by_side_and_errors(torch_cuda):
+    """Slabs interleaved inside each row (f[x][y][v], slab y): equals one
+    batch-contiguous solve; aliasing strides are rejected."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilderError
+    sb, orc = make(3, 500, PERIODIC, "sin")
+    n, B, nslab = sb.n, 24, 6
+    b = inputs.rhs(n, B * nslab, seed=61)
+    t = torch.from_numpy(b.copy()).cuda()
+    sb.solve_slabs_(t, B, B * nslab, nslab, B)
+    torch.cuda.synchronize()
+    assert rel_coef_error(t.cpu().numpy(), orc.solve(b)) <= TOL64
+    with pytest.raises(SplineBuilderError):
+        sb.solve_slabs_(t, B, B * nslab, nslab, B - 1)
+
+
+def test_c4m_middle_layout_matches_point_layout(torch_cuda):
+    """C4's second layout f[y][x][v] (x in the middle) via slabs gives the same
+    coefficients as the x-contiguous layout solved by the warp kernel."""
+    torch = torch_cuda
+    sb, orc = make(3, 1024, PERIODIC, "uniform")
+    n, Y, V = sb.n, 8, 256
+    b = inputs.rhs(n, Y * V, seed=62)                     # (n, Y*V)
+    mid = np.ascontiguousarray(b.reshape(n, Y, V).transpose(1, 0, 2))  # f[y][x][v]
+    t = torch.from_numpy(mid).cuda()
+    sb.solve_slabs_(t, V, V, Y, n * V)
+    pt = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()  # f[r][x]
+    sb.solve_(pt)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy().transpose(1, 0, 2).reshape(n, Y * V)
+    ref = orc.solve(b)
+    assert rel_coef_error(got, ref) <= TOL64
+    assert rel_coef_error(pt.cpu().numpy().T, ref) <= TOL64
+
+
+# ----------------------------------------- 2-D tensor product (solve_2d, f3)
+CASES_2D = [
+    # (dim-1 space, dim-2 space, grids)
+    ((3, 64, PERIODIC, "uniform"), (3, 48, PERIODIC, "uniform"), 5),
+    ((3, 200, PERIODIC, "sin"), (5, 150, GREVILLE, "sin"), 3),
+    ((5, 120, HERMITE, "jitter"), (4, 100, PERIODIC, "jitter"), 3),
+    ((4, 33, GREVILLE, "uniform"), (3, 1000, PERIODIC, "uniform"), 2),
+    ((3, 1024, PERIODIC, "uniform"), (3, 17, PERIODIC, "uniform"), 2),
+]
+
+
+def rel_grid_error(got, ref):
+    return float(max(np.abs(g - r).max() / np.abs(r).max() for g, r in zip(got, ref)))
+
+
+@pytest.mark.parametrize("c1,c2,G", CASES_2D, ids=[f"{a[0]}{a[2]}{a[1]}x{b[0]}{b[2]}{b[1]}" for a, b, _ in CASES_2D])
+def test_2d_parity(torch_cuda, c1, c2, G):
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import solve_2d_
+    sb1, o1 = make(*c1)
+    sb2, o2 = make(*c2)
+    F = inputs.rhs(sb1.n, G * sb2.n, seed=70).T.reshape(G, sb2.n, sb1.n).copy()
+    ref = oracle.solve_2d(o1, o2, F)
+    t = torch.from_numpy(F).cuda()
+    solve_2d_(sb1, sb2, t)
+    torch.cuda.synchronize()
+    assert rel_grid_error(t.cpu().numpy(), ref) <= TOL64
+    t32 = torch.from_numpy(F.astype(np.float32)).cuda()
+    solve_2d_(sb1, sb2, t32)
+    torch.cuda.synchronize()
+    ref32 = oracle.solve_2d(o1, o2, F.astype(np.float32).astype(np.float64))
+    assert rel_grid_error(t32.cpu().numpy(), ref32) <= TOL32
+
+
+def test_2d_full_size_chunked_sampled(torch_cuda):
+    """C6 shape (1024 x 1024 grids, 16 of them: 128 MB, several L2 chunks):
+    sampled grids against the oracle, interpolation property on one grid."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import solve_2d_
+    sb1, o1 = make(3, 1024, PERIODIC, "uniform")
+    sb2, o2 = make(3, 1024, PERIODIC, "uniform")
+    G = 16
+    F = inputs.rhs(1024, G * 1024, seed=71).T.reshape(G, 1024, 1024).copy()
+    t = torch.from_numpy(F).cuda()
+    solve_2d_(sb1, sb2, t)
+    torch.cuda.synchronize()
+    out = t.cpu().numpy()
+    for g in (0, 7, 15):
+        ref = oracle.solve_2d(o1, o2, F[g])
+        assert rel_grid_error(out[g:g + 1], ref[None]) <= TOL64
+    # A1 C A2^T = F on grid 3
+    A1, A2 = o1.matrix(), o2.matrix()
+    res = np.abs(A2 @ out[3] @ A1.T - F[3]).max() / np.abs(F[3]).max()
+    assert res <= 1e-12

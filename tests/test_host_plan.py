@@ -151,3 +151,24 @@ def test_hermite_rejects_derivative_rows_in_q():
     from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilderError
     with pytest.raises(SplineBuilderError):
         host(5, 996, HERMITE, "sin", split=(1, 1))
+
+
+MIXED = [(p, N, lo, hi, kind) for p in (1, 2, 3, 4, 5) for (lo, hi) in ((HERMITE, GREVILLE), (GREVILLE, HERMITE))
+         for N, kind in ((60, "uniform"), (995, "sin"))]
+
+
+@pytest.mark.parametrize("case", MIXED, ids=[f"p{c[0]}-N{c[1]}-{c[2]}{c[3]}-{c[4]}" for c in MIXED])
+def test_mixed_bc_host_plan_matches_oracle(case):
+    """Mixed ends (NEXT row f4): the plan's split keeps every derivative row in
+    delta and reproduces the oracle."""
+    p, N, lo, hi, kind = case
+    bc = inputs.bc_mixed(lo, hi)
+    nlo, nhi = inputs.n_hermite_rows(p, bc)
+    npts = N + p - nlo - nhi
+    sb, x = host(p, npts, bc, kind)
+    inf = sb.info()
+    assert inf["n_cells"] == N and inf["nbasis"] == N + p
+    assert inf["split_lo"] >= nlo and inf["split_hi"] >= nhi
+    o = Oracle(p, npts, bc, x)
+    b = inputs.rhs(o.n, 9, seed=3, degree=p, bc=bc)
+    assert rel_coef_error(sb.solve_cpu_plan_(b.copy()), o.solve(b)) < 1e-13

@@ -20,7 +20,12 @@ deg, npts, bc, mesh, B, dt, layout, desc = bench.WORKLOADS[args.workload]
 n = inputs.nbasis(deg, npts, bc)
 sb = SplineBuilder(deg, npts, bc, inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh))
 x = torch.from_numpy(bench.make_rhs(deg, n, bc, B, 0, layout, dt)).cuda()
-for _ in range(args.n):
-    sb.solve_(x)
+if args.workload in bench.ADVECT:
+    sh = torch.from_numpy(bench.adv_shift(inputs.n_cells(deg, npts, bc), B)).cuda()
+    for _ in range(args.n):
+        sb.advect_(x, sh)
+else:
+    for _ in range(args.n):
+        sb.solve_(x)
 torch.cuda.synchronize()
 print("done", args.workload)
