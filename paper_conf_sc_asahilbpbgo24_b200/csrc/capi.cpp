@@ -189,7 +189,7 @@ int upload(spline_builder *h) {
     d.xe = (const double *)at(oXe); d.xi = (const double *)at(oXi);
     d.adv_uniform = P.adv_uniform ? 1 : 0; d.adv_invh = P.adv_invh; d.adv_q0 = P.adv_q0;
     d.adv_rcp = (const double *)at(oRcp);
-    d.adv_tbl = (const int *)at(oTbl); d.adv_nbkt = (int)P.adv_tbl.size();
+    d.adv_tbl = (const int *)at(oTbl); d.adv_nbkt = (int)P.adv_tbl.size(); d.adv_steps = P.adv_steps;
     d.adv_bscale = P.xe.empty() ? 0.0 : (double)P.adv_tbl.size() / (P.xb[P.N] - P.xb[0]);
     d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
     d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);

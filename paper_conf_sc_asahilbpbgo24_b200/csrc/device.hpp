@@ -37,7 +37,7 @@ struct DevPlan {
     double adv_invh, adv_q0; // 1/h, (xi_0 - x_0)/h
     const double *adv_rcp;   // non-uniform: 1/(t_{m+w} - t_m) at [(m+p)*p + w-1], m in [-p, N+p), w = 1..p
     const int *adv_tbl;      // non-uniform: bucket b of [x_0, x_N) -> cell of its left edge (bucket <= min cell)
-    int adv_nbkt;
+    int adv_nbkt, adv_steps;
     double adv_bscale;       // adv_nbkt / (x_N - x_0)
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
     DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),

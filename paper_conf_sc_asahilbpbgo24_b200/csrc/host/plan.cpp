@@ -9,6 +9,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <random>
@@ -569,17 +570,31 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         P.adv_uniform = dev <= 2.3e-16 * xmax;
         P.adv_invh = 1.0 / hu;
         P.adv_q0 = (P.xi[0] - P.xb[0]) / hu;
-        // bucket table: buckets no wider than the smallest cell, so the cell of a
-        // point is the bucket's cell or the next one
+        // bucket table: buckets no wider than the smallest cell (up to 8N of them);
+        // tbl[b] = cell holding the bucket's left edge minus a margin that covers
+        // the rounding of b = floor((x - x_0) * scale) on the device, so the true
+        // cell is tbl[b] + 0..adv_steps, found by adv_steps branch-free steps
         {
             double hmin = Lp;
             for (int c = 0; c < N; ++c) hmin = std::min(hmin, P.xb[c + 1] - P.xb[c]);
-            const int MT = (int)std::min<double>(8.0 * N, std::ceil(Lp / hmin * (1.0 + 1e-12)));
-            P.adv_tbl.resize(std::max(MT, 1));
-            for (int b = 0, c = 0; b < (int)P.adv_tbl.size(); ++b) {
-                const double x = P.xb[0] + b * (Lp / P.adv_tbl.size());
-                while (c + 1 < N && P.xb[c + 1] <= x) ++c;
-                P.adv_tbl[b] = c;
+            const int MT = std::max(1, (int)std::min<double>(8.0 * N, std::ceil(Lp / hmin * (1.0 + 1e-12))));
+            const double w = Lp / MT, margin = 1e-9 * w;
+            auto cell_of = [&](double x) {  // t_c <= x < t_{c+1}, clamped to [0, N)
+                int lo = 0, hi = N - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) / 2;
+                    if (P.xb[mid] <= x) lo = mid;
+                    else hi = mid - 1;
+                }
+                return lo;
+            };
+            P.adv_tbl.resize(MT);
+            P.adv_steps = 0;
+            for (int b = 0; b < MT; ++b) {
+                const int lo = cell_of(P.xb[0] + b * w - margin);
+                const int hi = cell_of(P.xb[0] + (b + 1) * w + margin);
+                P.adv_tbl[b] = lo;
+                P.adv_steps = std::max(P.adv_steps, hi - lo);
             }
         }
         // reciprocal knot differences 1/(t_{m+w} - t_m), m in [-p, N+p), w = 1..p:
@@ -648,7 +663,7 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
     for (auto &c : cands) {
         SplitResult r = try_split(P, c.first, c.second);
         if (r.code) { why = r.msg; why_code = r.code; continue; }
-        build_segplan(P, P.seg[0], 36);
+        build_segplan(P, P.seg[0], 36);  // tile kernel fp64 / fp32 (instantiated lengths)
         build_segplan(P, P.seg[1], 72);
         {   // warp-per-RHS kernel: odd L (conflict-free smem transpose), S <= 32
             const int need = std::max(P.K, (P.nQ + 31) / 32);

@@ -34,6 +34,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <mutex>
+#include <set>
+#include <utility>
 #include <type_traits>
 #include <cstdio>
 #include <cstring>
@@ -43,8 +46,23 @@
 namespace sb {
 
 enum Loader { LOAD_DIRECT = 0, LOAD_TMA = 1 };
+
+// shared-memory layout of the non-uniform advection geometry (doubles from
+// off_geo; every array 16-B aligned for the bulk copies):
+//   xe[N+2p+1] (t_c at xe[c+p]) | xi[n] | rcp[(N+2p) p] | bucket table (int)
+struct GeoLayout {
+    int o_xi, o_rc, o_tbl, total_doubles;
+    __host__ __device__ GeoLayout(const DevPlan &P) {
+        auto even = [](int x) { return (x + 1) & ~1; };
+        o_xi = even(P.N + 2 * P.p + 1);
+        o_rc = o_xi + even(P.n);
+        o_tbl = o_rc + even((P.N + 2 * P.p) * P.p);
+        total_doubles = o_tbl + (P.adv_nbkt + 1) / 2 + 2;
+    }
+};
 constexpr int NBOXMAX = 8;
-constexpr int WB_FRONT = 4;  // warp kernel: elements in front of each row buffer (advection wrap pad)
+constexpr int WB_FRONT = 4;
+constexpr int WARP_MAX_WARPS = 16;  // warp kernel: <= 16 warps per block / per SM (128 registers each)  // warp kernel: elements in front of each row buffer (advection wrap pad)
 constexpr int TILE_MAX_THREADS = 512;  // <= 15 compute warps + 1 corner/producer warp: 4 warps per
                                        // SM sub-partition keeps the 128-register budget
 
@@ -118,10 +136,6 @@ __device__ __forceinline__ void named_bar(int id, int count) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
 
-template <typename T>
-__device__ __forceinline__ void copy_words(T *dst, const T *src, int count, int tid, int nthreads) {
-    for (int i = tid; i < count; i += nthreads) dst[i] = src[i];
-}
 
 template <typename T> struct Vec2;
 template <> struct Vec2<double> { using type = double2; };
@@ -273,34 +287,69 @@ __device__ __forceinline__ void getrs_small(C *x1, const C *lu, const int *piv, 
     }
 }
 
-// stage the constants of one segment plan + the corner data into shared memory
+// Stage the constants of one segment plan + the corner data (+ the advection
+// geometry) into shared memory with bulk async copies (cp.async.bulk, one
+// instruction per array, completion on one mbarrier) instead of a
+// load/store loop: the copies stream at L2 bandwidth and cost the CTA a
+// single wait.  Every array starts 16-B aligned in the blob and in shared
+// memory and its size is rounded up to 16 B (the blob pads each array).
+struct StageList {
+    static constexpr int MAXN = 24;
+    void *dst[MAXN];
+    const void *src[MAXN];
+    uint32_t bytes[MAXN];
+    int n = 0;
+    uint32_t total = 0;
+    __device__ __forceinline__ void add(void *d, const void *sr, size_t nb) {
+        const uint32_t b16 = (uint32_t)((nb + 15) & ~(size_t)15);
+        if (b16 == 0) return;
+        dst[n] = d; src[n] = sr; bytes[n] = b16; ++n;
+        total += b16;
+    }
+};
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *mbar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(mbar))
+                 : "memory");
+}
+
+// one thread: arm the barrier with the total and issue every copy
 template <typename C, int K>
-__device__ __forceinline__ void stage_constants(const KParams &p, const DevSeg &G, unsigned char *smem, int tid,
-                                                int nthreads) {
+__device__ __forceinline__ void stage_constants_issue(const KParams &p, const DevSeg &G, unsigned char *smem,
+                                                      uint64_t *cbar) {
     constexpr int CI = sizeof(C) == 8 ? 0 : 1;
     const DevPlan &P = p.P;
     const int k = P.k, S = G.S;
-    const int nrec = K * G.nslots * G.LP;
-    copy_words(reinterpret_cast<C *>(smem + p.off_L), reinterpret_cast<const C *>(G.Lr[CI]), nrec, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_U), reinterpret_cast<const C *>(G.Ur[CI]), nrec, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_dinv), reinterpret_cast<const C *>(G.dinv[CI]), G.nslots * G.LP,
-               tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_G), reinterpret_cast<const C *>(G.G[CI]), S * K * K, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_H), reinterpret_cast<const C *>(G.H[CI]), S * K * K, tid, nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_lamptr), P.lam_ptr, k + 1, tid, nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_lamc), P.lam_c, P.lam_nnz, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_lamv), reinterpret_cast<const C *>(P.lam_v[CI]), P.lam_nnz, tid,
-               nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_gamr), P.gam_r, P.gam_nnz, tid, nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_gamc), P.gam_c, P.gam_nnz, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_gamv), reinterpret_cast<const C *>(P.gam_v[CI]), P.gam_nnz, tid,
-               nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_gptr), G.gptr, S + 1, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_dlu), reinterpret_cast<const C *>(P.dlu[CI]), k * k, tid, nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_dpiv), P.dpiv, k, tid, nthreads);
-    copy_words(reinterpret_cast<C *>(smem + p.off_dscale), reinterpret_cast<const C *>(P.dscale[CI]), k, tid,
-               nthreads);
-    copy_words(reinterpret_cast<int *>(smem + p.off_drow), P.drow, k, tid, nthreads);
+    const size_t esz = sizeof(C);
+    const size_t nrec = (size_t)K * G.nslots * G.LP;
+    StageList L;
+    L.add(smem + p.off_L, G.Lr[CI], nrec * esz);
+    L.add(smem + p.off_U, G.Ur[CI], nrec * esz);
+    L.add(smem + p.off_dinv, G.dinv[CI], (size_t)G.nslots * G.LP * esz);
+    L.add(smem + p.off_G, G.G[CI], (size_t)S * K * K * esz);
+    L.add(smem + p.off_H, G.H[CI], (size_t)S * K * K * esz);
+    L.add(smem + p.off_lamptr, P.lam_ptr, (size_t)(k + 1) * 4);
+    L.add(smem + p.off_lamc, P.lam_c, (size_t)P.lam_nnz * 4);
+    L.add(smem + p.off_lamv, P.lam_v[CI], (size_t)P.lam_nnz * esz);
+    L.add(smem + p.off_gamr, P.gam_r, (size_t)P.gam_nnz * 4);
+    L.add(smem + p.off_gamc, P.gam_c, (size_t)P.gam_nnz * 4);
+    L.add(smem + p.off_gamv, P.gam_v[CI], (size_t)P.gam_nnz * esz);
+    L.add(smem + p.off_gptr, G.gptr, (size_t)(S + 1) * 4);
+    L.add(smem + p.off_dlu, P.dlu[CI], (size_t)k * k * esz);
+    L.add(smem + p.off_dpiv, P.dpiv, (size_t)k * 4);
+    L.add(smem + p.off_dscale, P.dscale[CI], (size_t)k * esz);
+    L.add(smem + p.off_drow, P.drow, (size_t)k * 4);
+    if (p.adv && !P.adv_uniform) {  // advection geometry: xe | xi | rcp | bucket table, each 16-B aligned
+        const GeoLayout gl(P);
+        double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);
+        L.add(sgeo, P.xe, (size_t)(P.N + 2 * P.p + 1) * 8);
+        L.add(sgeo + gl.o_xi, P.xi, (size_t)P.n * 8);
+        L.add(sgeo + gl.o_rc, P.adv_rcp, (size_t)(P.N + 2 * P.p) * P.p * 8);
+        L.add(sgeo + gl.o_tbl, P.adv_tbl, (size_t)P.adv_nbkt * 4);
+    }
+    mbar_arrive_expect_tx(cbar, L.total);
+    for (int i = 0; i < L.n; ++i) bulk_g2s(L.dst[i], L.src[i], L.bytes[i], cbar);
 }
 
 // ========================================================= tile kernel
@@ -373,12 +422,14 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         mbar_init(x1full + 1, R);
         mbar_init(cfull + 0, 1);
         mbar_init(cfull + 1, 1);
+        mbar_init(cfull + 2, 1);  // constants staged
         fence_mbar_init();
         if (LOADER == LOAD_TMA) prefetch_tmap(&tmap);
         if (use_cbox) prefetch_tmap(&tmap_c);
+        stage_constants_issue<C, K>(p, G, smem, cfull + 2);
     }
-    stage_constants<C, K>(p, G, smem, tid, blockDim.x);
     __syncthreads();
+    mbar_wait(cfull + 2, 0);
 
     if (warp == ncw) {
         // ===================== corner + producer warp (runs one tile ahead)
@@ -781,44 +832,48 @@ template <typename C, typename T, int PD>
 __device__ __forceinline__ void advect_row_nu(const DevPlan &P, const double *sgeo, const C *coef, T *g,
                                               int64_t ps, double sh, int lane) {
     const int N = P.N;
-    const double *xe = sgeo + PD;               // xe[c] = t_c, c in [-PD, N+PD]
-    const double *xi = sgeo + N + 2 * PD + 1;   // interpolation points (n = N)
-    const double *rc = xi + N + PD * PD;        // rc[m*PD + w-1] = 1/(t_{m+w} - t_m), m in [-PD, N+PD)
-    const int *tbl = reinterpret_cast<const int *>(rc + (N + PD) * PD);
+    const GeoLayout gl(P);
+    const double *xe = sgeo + PD;                  // xe[c] = t_c, c in [-PD, N+PD]
+    const double *xi = sgeo + gl.o_xi;             // interpolation points (n = N)
+    const double *rc = sgeo + gl.o_rc + PD * PD;   // rc[m*PD + w-1] = 1/(t_{m+w} - t_m), m in [-PD, N+PD)
+    const int *tbl = reinterpret_cast<const int *>(sgeo + gl.o_tbl);
     const int MT = P.adv_nbkt;
     const double x0 = xe[0], xN = xe[N], Lp = xN - x0, invLp = 1.0 / Lp, bscale = P.adv_bscale;
     double shr = sh - floor(sh * invLp) * Lp;  // sh mod L, in [0, L)
     if (shr >= Lp) shr -= Lp;
     if (shr < 0.0) shr += Lp;
-    auto locate = [&](double x) {  // t_c <= x < t_{c+1}
+    const int nsteps = P.adv_steps;
+    auto locate = [&](double x) {  // t_c <= x < t_{c+1}: bucket, then nsteps branch-free steps
         int c = tbl[min(max((int)((x - x0) * bscale), 0), MT - 1)];
-        c += (x >= xe[c + 1]);
-        if (x < xe[c] || x >= xe[c + 1]) {  // rounding at a bucket edge: walk
-            while (c > 0 && x < xe[c]) --c;
-            while (c + 1 < N && x >= xe[c + 1]) ++c;
-        }
+        for (int q = 0; q < nsteps; ++q) c += (x >= xe[c + 1]);
         return c;
     };
+    // feet: xi_j in [x_0, x_N), shr in [0, L) -> one conditional wrap (x_N itself maps to x_0)
     auto foot = [&](int j) {
         double x = xi[j] - shr;
         if (x < x0) x += Lp;
         if (x >= xN) x -= Lp;
-        return (x >= x0 && x < xN) ? x : x0;
+        return x;
     };
-    for (int j0 = lane; j0 < N; j0 += 64) {
-        const int j1 = j0 + 32;
-        const bool v1 = j1 < N;
-        const double xa = foot(j0), xb = foot(v1 ? j1 : j0);
-        const int ca = locate(xa), cb = locate(xb);
+    // software pipeline: the cells of the next pair of points are located while
+    // the current pair is evaluated
+    int j0 = lane;
+    double xa = foot(min(j0, N - 1)), xb = foot(min(j0 + 32, N - 1));
+    int ca = locate(xa), cb = locate(xb);
+    for (; j0 < N; j0 += 64) {
+        const int j1 = j0 + 32, jn = j0 + 64;
+        const double xan = foot(min(jn, N - 1)), xbn = foot(min(jn + 32, N - 1));
+        const int can = locate(xan), cbn = locate(xbn);
         const C ya = nu_value<C, PD>(xa, ca, xe, coef, rc);
         const C yb = nu_value<C, PD>(xb, cb, xe, coef, rc);
         __stcs(g + (int64_t)j0 * ps, (T)ya);
-        if (v1) __stcs(g + (int64_t)j1 * ps, (T)yb);
+        if (j1 < N) __stcs(g + (int64_t)j1 * ps, (T)yb);
+        xa = xan; xb = xbn; ca = can; cb = cbn;
     }
 }
 
 template <typename T, int K, int L, bool BULK, bool ADV>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
     sb_warp_kernel(const __grid_constant__ KParams p) {
     using C = T;
     extern __shared__ __align__(1024) unsigned char smem[];
@@ -830,22 +885,21 @@ __global__ void __launch_bounds__(256)
     const int nwarps = blockDim.x >> 5;
 
     uint64_t *wbar = reinterpret_cast<uint64_t *>(smem + p.off_mbar) + 2 * warp;  // 2 per warp
+    uint64_t *cbar = reinterpret_cast<uint64_t *>(smem + p.off_mbar) + 2 * WARP_MAX_WARPS;  // constants staged
     if (BULK && lane == 0) {
         mbar_init(wbar, 1);
         mbar_init(wbar + 1, 1);
         fence_mbar_init();
     }
-    stage_constants<C, K>(p, G, smem, tid, blockDim.x);
-    // advect, non-uniform: xe[N+2p+1] | xi[n] | rcp[(N+2p) p] | bucket table (int)
-    double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);
-    if (ADV && !P.adv_uniform) {
-        copy_words(sgeo, P.xe, P.N + 2 * P.p + 1, tid, blockDim.x);
-        copy_words(sgeo + P.N + 2 * P.p + 1, P.xi, n, tid, blockDim.x);
-        copy_words(sgeo + P.N + 2 * P.p + 1 + n, P.adv_rcp, (P.N + 2 * P.p) * P.p, tid, blockDim.x);
-        copy_words(reinterpret_cast<int *>(sgeo + P.N + 2 * P.p + 1 + n + (P.N + 2 * P.p) * P.p), P.adv_tbl,
-                   P.adv_nbkt, tid, blockDim.x);
+    if (tid == 0) {
+        mbar_init(cbar, 1);
+        fence_mbar_init();
+        stage_constants_issue<C, K>(p, G, smem, cbar);
     }
+    // advect, non-uniform geometry (GeoLayout): xe | xi | rcp | bucket table
+    const double *sgeo = reinterpret_cast<const double *>(smem + p.off_geo);
     __syncthreads();
+    mbar_wait(cbar, 0);
 
     const C *sL = reinterpret_cast<const C *>(smem + p.off_L);
     const C *sU = reinterpret_cast<const C *>(smem + p.off_U);
@@ -1131,6 +1185,30 @@ int launch_warp_adv_f64(int K, int L, const KParams &kp, int grid, cudaStream_t 
 int launch_warp_adv_f32(int K, int L, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 int launch_serial(int dtype, int K, const KParams &kp, int grid, cudaStream_t st, char *err, int errlen);
 
+// Raise a kernel's dynamic shared-memory limit once per device (the attribute
+// call costs microseconds; small batches are launch-bound).  The limit is set
+// to the device maximum, which every launch's smem_total respects.
+template <typename F>
+inline cudaError_t smem_attr_once(F fn) {
+    static std::mutex mu;
+    static std::set<std::pair<const void *, int>> done;  // (kernel, device)
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const std::pair<const void *, int> key{reinterpret_cast<const void *>(fn), dev};
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        if (done.count(key)) return cudaSuccess;
+    }
+    int maxs = 0;
+    cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, maxs);
+    if (e == cudaSuccess) {
+        std::lock_guard<std::mutex> lk(mu);
+        done.insert(key);
+    }
+    return e;
+}
+
 inline int check_launch(const char *what, char *err, int errlen) {
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) {
@@ -1144,8 +1222,7 @@ template <typename T, int K, int L, int R, int LOADER>
 int launch_tile(const KParams &kp, const CUtensorMap *tm, int grid, int threads, cudaStream_t st, char *err,
                 int errlen) {
     auto fn = sb_tile_kernel<T, K, L, R, tile_nv(sizeof(T)), LOADER>;
-    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total) != cudaSuccess)
-        return check_launch("cudaFuncSetAttribute(tile)", err, errlen);
+    if (smem_attr_once(fn) != cudaSuccess) return check_launch("cudaFuncSetAttribute(tile)", err, errlen);
     fn<<<grid, threads, kp.smem_total, st>>>(kp, tm[0], tm[1]);
     return check_launch("tile kernel launch", err, errlen);
 }
@@ -1166,8 +1243,7 @@ int tile_K(int K, const KParams &kp, const CUtensorMap *tm, int grid, int thread
 template <typename T, int K, int L, bool ADV>
 int launch_warp1(const KParams &kp, int grid, cudaStream_t st, char *err, int errlen) {
     auto fn = kp.bulk ? sb_warp_kernel<T, K, L, true, ADV> : sb_warp_kernel<T, K, L, false, ADV>;
-    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kp.smem_total) != cudaSuccess)
-        return check_launch("cudaFuncSetAttribute(warp)", err, errlen);
+    if (smem_attr_once(fn) != cudaSuccess) return check_launch("cudaFuncSetAttribute(warp)", err, errlen);
     fn<<<grid, kp.warp_threads, kp.smem_total, st>>>(kp);
     return check_launch("warp kernel launch", err, errlen);
 }

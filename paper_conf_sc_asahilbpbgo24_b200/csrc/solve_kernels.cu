@@ -26,7 +26,7 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0) {
-    const size_t geo_bytes = (kp.adv && !P.adv_uniform) ? (size_t)(P.N + 2 * P.p + 1 + P.n + (P.N + 2 * P.p) * P.p) * 8 + (size_t)P.adv_nbkt * 4 : 0;
+    const size_t geo_bytes = (kp.adv && !P.adv_uniform) ? (size_t)GeoLayout(P).total_doubles * 8 : 0;
     size_t o = 0;
     auto take = [&](size_t bytes, size_t al) {
         o = align_up(o, al);
@@ -57,7 +57,7 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_drow = take((size_t)k * 4, 16);
     kp.off_cbuf = take((size_t)4 * cbox * R * esz, 128);
     kp.off_geo = take(geo_bytes, 16);
-    kp.off_mbar = take((2 * NBOXMAX + 4) * 8, 8);
+    kp.off_mbar = take((size_t)std::max(2 * NBOXMAX + 5, 2 * WARP_MAX_WARPS + 1) * 8, 8);  // tile: boxes; warp: 2 per warp; + constants
     kp.smem_total = (int)align_up(o, 16);
     return kp.smem_total;
 }
@@ -101,8 +101,8 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         return e ? atoi(e) : -1;
     }();
     struct Cand { bool bulk; int wpb; };
-    const Cand cands[] = {{true, 4}, {true, 2}, {true, 1}, {true, 8}, {true, 6}, {true, 3},
-                          {false, 8}, {false, 6}, {false, 4}, {false, 2}, {false, 1}};
+    const Cand cands[] = {{true, 4}, {true, 2}, {true, 1}, {true, 8}, {true, 6}, {true, 3}, {true, 12}, {true, 16},
+                          {false, 8}, {false, 6}, {false, 4}, {false, 2}, {false, 1}, {false, 12}, {false, 16}};
     const int out_row = (kp.adv && P.adv_uniform) ? 1 : 0;  // uniform advection writes via an output row
     int best = -1, best_score = 0;
     for (int ci = 0; ci < (int)(sizeof(cands) / sizeof(cands[0])); ++ci) {
@@ -112,7 +112,7 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         KParams t = kp;
         layout_smem(t, P, G, 1, esz, (size_t)c.wpb * ((c.bulk ? 2 : 1) + out_row) * kp.wbuf_pitch * esz);
         if (t.smem_total > max_smem) continue;
-        const int per_sm = std::min(16 / c.wpb, (int)(228 * 1024 / (t.smem_total + 1024)));
+        const int per_sm = std::min(WARP_MAX_WARPS / c.wpb, (int)(228 * 1024 / (t.smem_total + 1024)));
         // the bulk pipeline (double-buffered rows) is worth 1.5x the warps
         // (measured: C4 bulk 12 warps/SM 0.378 ms vs plain 16 warps 0.396 ms)
         const int score = c.wpb * std::max(per_sm, 1) * (c.bulk ? 3 : 2);
@@ -137,7 +137,7 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
     }
     const int wpb = kp.warp_threads / 32;
-    const int per_sm = std::max(1, std::min(16 / wpb, (int)(228 * 1024 / (kp.smem_total + 1024))));
+    const int per_sm = std::max(1, std::min(WARP_MAX_WARPS / wpb, (int)(228 * 1024 / (kp.smem_total + 1024))));
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + wpb - 1) / wpb, (int64_t)num_sms * per_sm));
     // round L up to an instantiated odd length (the plan chose the smallest odd L >= nQ/32)
     if (a.dtype == 0) return launch_warp_f64(P.K, G.L, kp, grid, a.stream, err, errlen);
@@ -164,8 +164,12 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     const size_t esz = a.dtype == 0 ? 8 : 4;
     int dev = 0;
     cudaGetDevice(&dev);
-    int max_smem = 0;
-    cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    static int max_smem_dev[64] = {0};  // per device, queried once
+    int max_smem = dev >= 0 && dev < 64 ? max_smem_dev[dev] : 0;
+    if (!max_smem) {
+        cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        if (dev >= 0 && dev < 64) max_smem_dev[dev] = max_smem;
+    }
 
     // point-contiguous / general strided layouts and the advection step: warp-per-RHS kernel
     if (a.bstride != 1 || a.shift) return launch_warp(P, a, num_sms, max_smem, err, errlen);

@@ -15,8 +15,11 @@ from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, inputs  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="C2")
 ap.add_argument("--n", type=int, default=3)
+ap.add_argument("--degree", type=int, default=None, help="override the workload's degree (periodic workloads)")
 args = ap.parse_args()
 deg, npts, bc, mesh, B, dt, layout, desc = bench.WORKLOADS[args.workload]
+if args.degree:
+    deg = args.degree
 n = inputs.nbasis(deg, npts, bc)
 sb = SplineBuilder(deg, npts, bc, inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh))
 x = torch.from_numpy(bench.make_rhs(deg, n, bc, B, 0, layout, dt)).cuda()

@@ -37,16 +37,22 @@ PAPER_A100 = {("uniform", 3): 268.6, ("uniform", 4): 252.6, ("uniform", 5): 251.
 
 
 def time_launches(fn, x, pristine, steps, warmup):
+    """ms per launch: `steps` launches captured in one CUDA graph and replayed
+    (Python's per-call overhead would otherwise dominate the small batches)."""
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     for _ in range(warmup):
         fn(x)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for _ in range(steps):
+            fn(x)
     x.copy_(pristine)
     flush.fill_(1)
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
     s.record()
-    for _ in range(steps):
-        fn(x)
+    g.replay()
     e.record()
     torch.cuda.synchronize()
     return s.elapsed_time(e) / steps
@@ -94,9 +100,11 @@ def main():
                 v = -1.0 + 2.0 * np.arange(nv) / nv
                 shift = torch.from_numpy(v * 2.5 / nx).cuda()
                 ms = time_launches(lambda t: sb.advect_(t, shift), x, pristine, args.steps, args.warmup)
+                ms_solve = time_launches(sb.solve_, x, pristine, args.steps, args.warmup)
                 emit({"figure": "2", "mesh": "uniform" if mesh == "uniform" else "non-uniform (sin map)",
                       "degree": p, "nx": nx, "nv": nv, "ms": ms, "glups": nx * nv * 1e-9 / (ms / 1e3),
-                      "gbs_16B": 16.0 * nx * nv / (ms / 1e3) / 1e9, "layout": "point-contiguous (x fastest)"})
+                      "gbs_16B": 16.0 * nx * nv / (ms / 1e3) / 1e9, "layout": "point-contiguous (x fastest)",
+                      "ms_build_only": ms_solve, "q_band": [sb.info()["q_kl"], sb.info()["q_ku"]]})
                 del x, pristine
     if out:
         out.close()
