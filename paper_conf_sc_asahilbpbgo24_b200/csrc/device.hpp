@@ -35,7 +35,7 @@ struct DevPlan {
     const double *xe, *xi;   // periodic extended knots t_c at xe[c+p] (N+2p+1), n row positions
     int adv_uniform;         // uniform periodic mesh: Algorithm 2's evaluation is a per-row stencil
     double adv_invh, adv_q0; // 1/h, (xi_0 - x_0)/h
-    const double *adv_rcp;   // non-uniform: 1/(t_{m+w} - t_m) at [(m+p)*p + w-1], m in [-p, N+p), w = 1..p
+    const double *adv_rcp;   // non-uniform: 1/(t_{m+w} - t_m) at [(m+p)*(p|1) + w-1], m in [-p, N+p), w = 1..p
     const int *adv_tbl;      // non-uniform: bucket b of [x_0, x_N) -> cell of its left edge (bucket <= min cell)
     int adv_nbkt, adv_steps;
     double adv_bscale;       // adv_nbkt / (x_N - x_0)

@@ -600,10 +600,11 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         // reciprocal knot differences 1/(t_{m+w} - t_m), m in [-p, N+p), w = 1..p:
         // the denominators of de Boor's recursion depend on the knots only, so the
         // non-uniform evaluation multiplies instead of dividing
-        P.adv_rcp.assign((size_t)(N + 2 * p) * p, 0.0);
+        const int RS = p | 1;  // odd row stride: lanes at consecutive cells hit distinct banks
+        P.adv_rcp.assign((size_t)(N + 2 * p) * RS, 0.0);
         for (int m = -p; m < N + p; ++m)
             for (int w = 1; w <= p; ++w)
-                if (m + w <= N + p) P.adv_rcp[(size_t)(m + p) * p + (w - 1)] = 1.0 / (P.xe[m + w + p] - P.xe[m + p]);
+                if (m + w <= N + p) P.adv_rcp[(size_t)(m + p) * RS + (w - 1)] = 1.0 / (P.xe[m + w + p] - P.xe[m + p]);
     }
     // equilibrated sparse rows: rowscale * (d^deriv B_j)(point)
     P.A.assign(n, SparseRow());

@@ -48,7 +48,7 @@ struct Plan {
     double adv_invh = 0.0, adv_q0 = 0.0;  // 1/h and (xi_0 - x_0)/h
     int adv_steps = 0;              // forward steps from the bucket's cell to the point's cell (<= 2 typically)
     std::vector<int> adv_tbl;       // periodic: buckets of [x_0, x_N) no wider than the smallest cell -> cell
-    std::vector<double> adv_rcp;    // periodic: 1/(t_{m+w} - t_m) at [(m+p)*p + w-1], m in [-p, N+p), w = 1..p
+    std::vector<double> adv_rcp;    // periodic: 1/(t_{m+w} - t_m) at [(m+p)*(p|1) + w-1], m in [-p, N+p), w = 1..p
     std::vector<SparseRow> A;       // equilibrated collocation matrix rows
     std::vector<double> rowscale;   // A_eq = diag(rowscale) * A_raw
     // ---- Schur split (Eq. 3)

@@ -56,7 +56,7 @@ struct GeoLayout {
         auto even = [](int x) { return (x + 1) & ~1; };
         o_xi = even(P.N + 2 * P.p + 1);
         o_rc = o_xi + even(P.n);
-        o_tbl = o_rc + even((P.N + 2 * P.p) * P.p);
+        o_tbl = o_rc + even((P.N + 2 * P.p) * (P.p | 1));
         total_doubles = o_tbl + (P.adv_nbkt + 1) / 2 + 2;
     }
 };
@@ -345,7 +345,7 @@ __device__ __forceinline__ void stage_constants_issue(const KParams &p, const De
         double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);
         L.add(sgeo, P.xe, (size_t)(P.N + 2 * P.p + 1) * 8);
         L.add(sgeo + gl.o_xi, P.xi, (size_t)P.n * 8);
-        L.add(sgeo + gl.o_rc, P.adv_rcp, (size_t)(P.N + 2 * P.p) * P.p * 8);
+        L.add(sgeo + gl.o_rc, P.adv_rcp, (size_t)(P.N + 2 * P.p) * (P.p | 1) * 8);
         L.add(sgeo + gl.o_tbl, P.adv_tbl, (size_t)P.adv_nbkt * 4);
     }
     mbar_arrive_expect_tx(cbar, L.total);
@@ -750,7 +750,8 @@ template <typename C, int PD>
 __device__ __forceinline__ C nu_value(double x, int c, const double *xe, const C *coef, const double *rc) {
     constexpr int s = (PD + 1) / 2;
     const double *tk = xe + c;       // tk[q] = t_{c+q}
-    const double *rk = rc + c * PD;  // rk[m*PD + w-1] = 1/(t_{c+m+w} - t_{c+m})
+    constexpr int RS = PD | 1;       // odd row stride of the reciprocal table (bank-conflict free)
+    const double *rk = rc + c * RS;  // rk[m*RS + w-1] = 1/(t_{c+m+w} - t_{c+m})
     double b[PD + 1];
     b[0] = 1.0;
 #pragma unroll
@@ -758,7 +759,7 @@ __device__ __forceinline__ C nu_value(double x, int c, const double *xe, const C
         double saved = 0.0;
 #pragma unroll
         for (int r = 0; r <= j; ++r) {
-            const double term = b[r] * rk[(r - j) * PD + j];  // 1/(t_{c+1+r} - t_{c-j+r})
+            const double term = b[r] * rk[(r - j) * RS + j];  // 1/(t_{c+1+r} - t_{c-j+r})
             b[r] = fma(tk[1 + r] - x, term, saved);
             saved = (x - tk[r - j]) * term;
         }
@@ -771,14 +772,13 @@ __device__ __forceinline__ C nu_value(double x, int c, const double *xe, const C
     return acc;
 }
 
-// One row of the advection step.
-// Uniform mesh: every foot xi_i - shift has the same local coordinate u, so
-// the weights are computed once per row and out[i] = sum_r w_r coef[i+off+r]
-// is a (p+1)-tap stencil.  Lane l owns the run of window starts
-// [l*M, l*M+M) (M odd: conflict-free smem strides) and slides a register
-// window along it: ~N + 32p shared loads per row instead of (p+1) N.
-template <typename C, int PD>
-__device__ __forceinline__ void advect_row(const DevPlan &P, const C *coef, C *out, double sh, int lane) {
+// One row of the advection step, uniform mesh: every foot xi_i - shift has
+// the same local coordinate u, so the p+1 weights are computed once per row
+// and out[i] = sum_r w_r coef[(i+off+r) mod N] is a (p+1)-tap stencil.  Lanes
+// take consecutive points (conflict-free shared loads; the row is padded past
+// N by the periodic wrap) and store straight to HBM, coalesced.
+template <typename C, typename T, int PD>
+__device__ __forceinline__ void advect_row(const DevPlan &P, const C *coef, T *g, int64_t ps, double sh, int lane) {
     constexpr int s = (PD + 1) / 2;
     const int N = P.N;
     const double q = P.adv_q0 - sh * P.adv_invh;  // foot of point 0, in cells from x_0
@@ -797,29 +797,15 @@ __device__ __forceinline__ void advect_row(const DevPlan &P, const C *coef, C *o
     c0 = c0 >= N ? c0 - N : (c0 < 0 ? c0 + N : c0);
     int off = c0 - PD + s;  // point i reads coef[i + off .. i + off + PD] (mod N)
     off = off < 0 ? off + N : (off >= N ? off - N : off);
-    const int M = ((N + 31) >> 5) | 1;
-    const int cbeg = lane * M;
-    if (cbeg >= N) return;
-    const int cend = min(cbeg + M, N);
-    C win[PD + 1];
-    int idx = cbeg;
-#pragma unroll
-    for (int r = 0; r < PD; ++r) {
-        win[r] = coef[idx];
-        idx = idx + 1 == N ? 0 : idx + 1;
-    }
-    int jr = cbeg - off;
-    jr = jr < 0 ? jr + N : jr;
-    for (int c = cbeg; c < cend; ++c) {
-        win[PD] = coef[idx];
-        idx = idx + 1 == N ? 0 : idx + 1;
+#pragma unroll 4
+    for (int i = lane; i < N; i += 32) {
+        int idx = i + off;
+        idx -= idx >= N ? N : 0;
+        const C *cw = coef + idx;
         C acc = C(0);
 #pragma unroll
-        for (int r = 0; r <= PD; ++r) acc = fma(w[r], win[r], acc);
-        out[jr] = acc;
-        jr = jr + 1 == N ? 0 : jr + 1;
-#pragma unroll
-        for (int r = 0; r < PD; ++r) win[r] = win[r + 1];
+        for (int r = 0; r <= PD; ++r) acc = fma(w[r], cw[r], acc);
+        __stcs(g + (int64_t)i * ps, (T)acc);
     }
 }
 
@@ -835,7 +821,7 @@ __device__ __forceinline__ void advect_row_nu(const DevPlan &P, const double *sg
     const GeoLayout gl(P);
     const double *xe = sgeo + PD;                  // xe[c] = t_c, c in [-PD, N+PD]
     const double *xi = sgeo + gl.o_xi;             // interpolation points (n = N)
-    const double *rc = sgeo + gl.o_rc + PD * PD;   // rc[m*PD + w-1] = 1/(t_{m+w} - t_m), m in [-PD, N+PD)
+    const double *rc = sgeo + gl.o_rc + PD * (PD | 1);  // rc[m*(PD|1) + w-1] = 1/(t_{m+w} - t_m), m in [-PD, N+PD)
     const int *tbl = reinterpret_cast<const int *>(sgeo + gl.o_tbl);
     const int MT = P.adv_nbkt;
     const double x0 = xe[0], xN = xe[N], Lp = xN - x0, invLp = 1.0 / Lp, bscale = P.adv_bscale;
@@ -917,10 +903,8 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
     const C *sdscale = reinterpret_cast<const C *>(smem + p.off_dscale);
     const int *sdrow = reinterpret_cast<const int *>(smem + p.off_drow);
     // per warp: row buffer(s) of WB_FRONT pad + n values + k spare for x1 (the
-    // advection pads the row on both sides); uniform advection: + an output row
-    const int nbuf = (BULK ? 2 : 1) + ((ADV && P.adv_uniform) ? 1 : 0);
-    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * nbuf * p.wbuf_pitch + WB_FRONT;
-    C *outrow = wbuf + (size_t)(BULK ? 2 : 1) * p.wbuf_pitch;  // ADV (uniform): the advected row
+    // advection pads the row on both sides with the periodic wrap)
+    C *wbuf = reinterpret_cast<C *>(smem + p.off_buf) + (size_t)warp * (BULK ? 2 : 1) * p.wbuf_pitch + WB_FRONT;
 
     const int s = lane;
     const bool active = s < S;
@@ -1039,22 +1023,20 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
         if (ADV) {
             // ---------- Algorithm 2: f(xi_i) <- S(xi_i - shift) while the coefficients are on chip
             const double sh = p.shift[rhs];
+            // wrap pads: rowbuf[-2..-1] = rowbuf[n-2..n-1], rowbuf[n..n+4] = rowbuf[0..4] (mod n)
+            __syncwarp();
+            if (lane < 2) rowbuf[lane - 2] = rowbuf[n - 1 - ((1 - lane) % n)];
+            else if (lane < 7) rowbuf[n + lane - 2] = rowbuf[(lane - 2) % n];
+            __syncwarp();
             if (P.adv_uniform) {
-                __syncwarp();
                 switch (P.p) {  // degrees 1..5 (the library's range)
-                    case 1: advect_row<C, 1>(P, rowbuf, outrow, sh, lane); break;
-                    case 2: advect_row<C, 2>(P, rowbuf, outrow, sh, lane); break;
-                    case 3: advect_row<C, 3>(P, rowbuf, outrow, sh, lane); break;
-                    case 4: advect_row<C, 4>(P, rowbuf, outrow, sh, lane); break;
-                    default: advect_row<C, 5>(P, rowbuf, outrow, sh, lane); break;
+                    case 1: advect_row<C, T, 1>(P, rowbuf, g, ps, sh, lane); break;
+                    case 2: advect_row<C, T, 2>(P, rowbuf, g, ps, sh, lane); break;
+                    case 3: advect_row<C, T, 3>(P, rowbuf, g, ps, sh, lane); break;
+                    case 4: advect_row<C, T, 4>(P, rowbuf, g, ps, sh, lane); break;
+                    default: advect_row<C, T, 5>(P, rowbuf, g, ps, sh, lane); break;
                 }
-                res = outrow;
             } else {
-                // wrap pads: rowbuf[-2..-1] = rowbuf[n-2..n-1], rowbuf[n..n+2] = rowbuf[0..2]
-                __syncwarp();
-                if (lane < 2) rowbuf[lane - 2] = rowbuf[n - 2 + lane];
-                else if (lane < 5) rowbuf[n + lane - 2] = rowbuf[lane - 2];
-                __syncwarp();
                 switch (P.p) {
                     case 1: advect_row_nu<C, T, 1>(P, sgeo, rowbuf, g, ps, sh, lane); break;
                     case 2: advect_row_nu<C, T, 2>(P, sgeo, rowbuf, g, ps, sh, lane); break;
@@ -1062,8 +1044,8 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
                     case 4: advect_row_nu<C, T, 4>(P, sgeo, rowbuf, g, ps, sh, lane); break;
                     default: advect_row_nu<C, T, 5>(P, sgeo, rowbuf, g, ps, sh, lane); break;
                 }
-                direct = true;
             }
+            direct = true;
         }
         if (BULK && direct) {
             __syncwarp();  // every lane is done reading this row buffer

@@ -103,7 +103,7 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
     struct Cand { bool bulk; int wpb; };
     const Cand cands[] = {{true, 4}, {true, 2}, {true, 1}, {true, 8}, {true, 6}, {true, 3}, {true, 12}, {true, 16},
                           {false, 8}, {false, 6}, {false, 4}, {false, 2}, {false, 1}, {false, 12}, {false, 16}};
-    const int out_row = (kp.adv && P.adv_uniform) ? 1 : 0;  // uniform advection writes via an output row
+    const int out_row = 0;  // the advection stores straight to HBM (no output row buffer)
     int best = -1, best_score = 0;
     for (int ci = 0; ci < (int)(sizeof(cands) / sizeof(cands[0])); ++ci) {
         const Cand &c = cands[ci];
