@@ -76,6 +76,13 @@ WORKLOADS = {
 }
 
 
+# Practical in-place streaming ceilings on this pool (no-math read-modify-write
+# kernels with the solver's access patterns, tools/stream_probe*.cu;
+# profiles/r01/stream_probe*_session2.txt): batch-contiguous 16/32-RHS TMA tiles
+# + st.cs writes, and flat contiguous rows (the point layout).
+STREAM_CEILING_GBS = {"batch": 5681.0, "slabs": 5681.0, "point": 6372.0}
+
+
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -531,6 +538,8 @@ def main():
             done += m
         barrier()
     total_ms = float(sum(s_.elapsed_time(e_) for s_, e_ in zip(starts, ends)))
+    chunk_steps = [min(CHUNK, args.steps - c * CHUNK) for c in range(nchunks)]
+    per_chunk = [s_.elapsed_time(e_) / m for s_, e_, m in zip(starts, ends, chunk_steps)]  # ms per step
     t_tensor = torch.tensor([total_ms, total_ms / args.steps], device="cuda", dtype=torch.float64)
     if ws > 1:
         dist.all_reduce(t_tensor, op=dist.ReduceOp.MAX)
@@ -605,9 +614,13 @@ def main():
                        "inputs": "device Philox (inputs.rhs_device)" if on_device else "host Philox (inputs.rhs)",
                        "launch": "python per step" if args.no_graph else "CUDA graph of 40 launches, replayed",
                        "parallelism": f"dp{ws} (RHS shards)"},
+            "ms_per_step_median": float(np.median(per_chunk)), "ms_per_step_best": float(min(per_chunk)),
+            "timed_chunks": len(per_chunk),
             "achieved_gbs": achieved, "pct_of_8tbs": achieved / 8000.0,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": load_traffic(args.workload),
+                         "stream_ceiling_gbs": STREAM_CEILING_GBS[layout],
+                         "frac_of_stream_ceiling": achieved / STREAM_CEILING_GBS[layout],
                          "peak_kind": peak_kind, "kernel_ms": kern_avg_ms,
                          "algorithmic_bytes_per_launch": alg_bytes},
             "clocks": clk.summary(),

@@ -16,6 +16,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="C2")
 ap.add_argument("--n", type=int, default=3)
 ap.add_argument("--degree", type=int, default=None, help="override the workload's degree (periodic workloads)")
+ap.add_argument("--solve", action="store_true", help="plain solve even for an advection workload")
 args = ap.parse_args()
 deg, npts, bc, mesh, B, dt, layout, desc = bench.WORKLOADS[args.workload]
 if args.degree:
@@ -23,7 +24,7 @@ if args.degree:
 n = inputs.nbasis(deg, npts, bc)
 sb = SplineBuilder(deg, npts, bc, inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh))
 x = torch.from_numpy(bench.make_rhs(deg, n, bc, B, 0, layout, dt)).cuda()
-if args.workload in bench.ADVECT:
+if args.workload in bench.ADVECT and not args.solve:
     sh = torch.from_numpy(bench.adv_shift(inputs.n_cells(deg, npts, bc), B)).cuda()
     for _ in range(args.n):
         sb.advect_(x, sh)
