@@ -9,7 +9,8 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libsplinebuilder.so")
+# SB_LIB_PATH: load another build of the same library (A/B experiments)
+LIB_PATH = os.environ.get("SB_LIB_PATH") or os.path.join(HERE, "libsplinebuilder.so")
 
 SB_PERIODIC, SB_GREVILLE, SB_HERMITE = 0, 1, 2
 SB_F64, SB_F32 = 0, 1

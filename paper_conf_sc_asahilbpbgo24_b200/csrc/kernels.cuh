@@ -248,9 +248,17 @@ __device__ __forceinline__ void bwd_local(C (&v)[L][NV], const C *fU, const C *f
     }
 }
 
-// backward correction chain c_i = -sum_m U'(i,i+1+m) c_{i+1+m}, c(a+L+m) = co[m];  x_i += c_i
-template <typename C, int K, int L, int NV, bool PAIRS>
-__device__ __forceinline__ void bwd_correct(C (&v)[L][NV], const C *fU, int ms, C (&co)[K][NV]) {
+// backward correction chain c_i = -sum_m U'(i,i+1+m) c_{i+1+m}, c(a+L+m) = co[m];  x_i += c_i.
+// STORE: row i is final once corrected, so it goes to HBM right there (one
+// NV-wide vector at dst + i*ps, rows i < nvalid): the stores trickle out under the chain's
+// FMA latency instead of leaving every warp of the tile in one burst.
+template <typename C, int K, int L, int NV, bool PAIRS, bool STORE = false, typename T = C>
+__device__ __forceinline__ void bwd_correct(C (&v)[L][NV], const C *fU, int ms, C (&co)[K][NV],
+                                            T *dst = nullptr, int64_t ps = 0, int nvalid = 0) {
+    using V = typename std::conditional<NV == 1, T,
+                                        typename std::conditional<sizeof(T) == 8, double2,
+                                                                  typename std::conditional<NV == 2, float2,
+                                                                                            float4>::type>::type>::type;
 #pragma unroll
     for (int i = L - (PAIRS ? 2 : 1); i >= 0; i -= (PAIRS ? 2 : 1)) {
         C u0[K], u1[K];
@@ -266,6 +274,13 @@ __device__ __forceinline__ void bwd_correct(C (&v)[L][NV], const C *fU, int ms, 
                 for (int m = K - 1; m > 0; --m) co[m][q] = co[m - 1][q];
                 co[0][q] = c;
                 v[i + h][q] += c;
+            }
+            if (STORE && i + h < nvalid) {
+                V w;
+                T *pw = reinterpret_cast<T *>(&w);
+#pragma unroll
+                for (int q = 0; q < NV; ++q) pw[q] = (T)v[i + h][q];
+                __stcs(reinterpret_cast<V *>(dst + (int64_t)(i + h) * ps), w);
             }
         }
     }
@@ -638,7 +653,13 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 for (int j = 0; j < K; ++j) sbbeg[(s * R + r0 + q) * K + j] = st[j][q];
         named_bar(1, nthr_c);  // B3
         // ---------- backward carry (true x at rows a+L..a+L+K-1) + correction chain
-        if (active && s < S - 1) {
+        // TMA path, band K >= 2: every row is stored from inside the chain as soon as
+        // it is final (the last segment runs the chain with zero carries, so there is
+        // one store path).  Measured: C3 Greville 0.403 -> 0.380 ms, Hermite 0.335 ->
+        // 0.326 ms; for K = 1 (C2) the chain is too short to hide the stores and the
+        // burst after it is faster (0.285 vs 0.314 ms).
+        constexpr bool FUSED = LOADER == LOAD_TMA && NV == 1 && K >= 2;
+        if (active && (FUSED || s < S - 1)) {
             C co[K][NV];
 #pragma unroll
             for (int m = 0; m < K; ++m)
@@ -660,13 +681,17 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
 #pragma unroll
                     for (int q = 0; q < NV; ++q) co[j][q] = nw[j][q];
             }
-            bwd_correct<C, K, L, NV, true>(v, fU, ms, co);
+            if constexpr (FUSED)
+                bwd_correct<C, K, L, NV, true, true, T>(v, fU, ms, co, gcol + (int64_t)(s_lo + a) * ps, ps,
+                                                        nlive > 0 ? min(L, nQ - a) : 0);
+            else
+                bwd_correct<C, K, L, NV, true>(v, fU, ms, co);
         }
         // ---------- store x0 straight from registers (one 16-B vector per row).
         // DIRECT mode: the corner warp reads b0 from HBM, so no row of this tile is
         // overwritten before x1 is done.
         if (LOADER == LOAD_DIRECT && k > 0) mbar_wait(x1full + (it & 1), (it >> 1) & 1);
-        if (nlive > 0) {
+        if (!FUSED && nlive > 0) {
             T *dst = gcol + (int64_t)(s_lo + a) * ps;
             if (LOADER == LOAD_TMA && nlive == NV && full_seg) {
 #pragma unroll
