@@ -40,7 +40,9 @@ def _newer(target: str, deps: list[str]) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, extra_flags: tuple = (), lib: str = LIB, build_dir: str = BUILD) -> str:
+    """extra_flags / lib / build_dir: diagnostic variants (e.g. -DSB_TRACE) built beside the shipped library."""
+    LIB, BUILD = lib, build_dir
     os.makedirs(BUILD, exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "spline_builder.h")]
     objs, jobs = [], []
@@ -55,7 +57,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
                    "-I" + os.path.join(CUDA_HOME, "include"), "-c", path, "-o", obj]
         else:
             cmd = [NVCC, *ARCH, "-std=c++17", "-O3", "-lineinfo", "-Xptxas", "-v", "-Xcompiler", "-fPIC",
-                   "--expt-relaxed-constexpr", "-c", path, "-o", obj]
+                   "--expt-relaxed-constexpr", *extra_flags, "-c", path, "-o", obj]
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
         jobs.append((cmd, obj, kind))

@@ -87,6 +87,32 @@ struct KParams {
     int adv, off_geo;                // advect flag; smem offset of xe[N+2p+1], xi[n], rcp[(N+2p) p] (fp64)
 };
 
+// SB_TRACE (diagnostic builds only, never the shipped library): lane 0 of
+// every warp of blocks < 4 records a timestamp at up to 9 points of its first
+// TR_TILES tiles into g_sb_trace[block][tile][warp][point] (tools/trace_tile.py).
+#ifdef SB_TRACE
+constexpr int TR_BLOCKS = 4, TR_TILES = 8, TR_WARPS = 16, TR_PTS = 9;
+static __device__ long long g_sb_trace[TR_BLOCKS * TR_TILES * TR_WARPS * TR_PTS];
+__device__ __forceinline__ long long sb_trace_clock() {
+#ifdef SB_TRACE_GLOBALTIMER
+    long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+#else
+    return clock64();
+#endif
+}
+#define SB_TR(pt)                                                                                          \
+    do {                                                                                                   \
+        if (lane == 0 && blockIdx.x < TR_BLOCKS && it < TR_TILES)                                          \
+            g_sb_trace[((blockIdx.x * TR_TILES + it) * TR_WARPS + warp) * TR_PTS + (pt)] = sb_trace_clock(); \
+    } while (0)
+#else
+#define SB_TR(pt) \
+    do {          \
+    } while (0)
+#endif
+
 // ------------------------------------------------------------- PTX helpers
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -465,6 +491,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
             const int slab = tile / p.tps, tb = tile - slab * p.tps;
             T *gs = gout + slab * p.slab_stride;
+            SB_TR(0);
             if (LOADER == LOAD_TMA) {
                 if (lane == 0) {
                     for (int c = 0; c < nbox; ++c) {
@@ -474,12 +501,14 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                     }
                     if (use_cbox && tile + (int)gridDim.x < p.ntiles) issue_cbox(tile + gridDim.x, (it + 1) & 1);
                 }
+                SB_TR(8);
                 if (use_cbox) mbar_wait(cfull + (it & 1), (it >> 1) & 1);
                 else
                     for (int c = 0; c < nbox; ++c) mbar_wait(full + c, it & 1);
             } else if (it > 0) {
                 mbar_wait(empty + 0, (it - 1) & 1);  // all compute warps finished tile it-1
             }
+            SB_TR(2);
             const T *cb = cbuf + (size_t)(it & 1) * 2 * cbox * R;
             const int64_t ccol = (int64_t)tb * R + rr;
             const bool clive = ccol < p.batch;
@@ -510,11 +539,13 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 for (int off = R; off < 32; off *= 2) acc += __shfl_xor_sync(0xffffffffu, acc, off);
                 if (part == 0) x1[d] = acc;
             }
+            SB_TR(3);
             if (part == 0 && k > 0) {
                 getrs_small(x1, sdlu, sdpiv, k);
                 if (clive)
                     for (int d = 0; d < k; ++d) __stcs(gs + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
             }
+            SB_TR(1);
             __syncwarp();
             if (part == 0) mbar_arrive(x1full + (it & 1));
             if (lane == 0) {
@@ -558,9 +589,11 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         const int nlive = active ? (int)max((int64_t)0, min((int64_t)NV, p.batch - col0)) : 0;
         T *gcol = gout + slab * p.slab_stride + col0 * p.bstride;
         C v[L][NV];
+        SB_TR(0);
         // ---------- own segment of b0 into registers
         if (LOADER == LOAD_TMA) {
             for (int c = c_lo; c <= c_hi; ++c) mbar_wait(full + c, it & 1);
+            SB_TR(8);
             const T *src = buf + (size_t)(s_lo + a) * R + r0;
             if (full_seg) {
 #pragma unroll
@@ -595,6 +628,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 for (int q = 0; q < NV; ++q)
                     v[i][q] = (q < nlive && a + i < nQ) ? (C)__ldcs(src + (int64_t)i * ps + q * p.bstride) : C(0);
         }
+        SB_TR(1);
         // ---------- b0 -= gamma x1 (only segments holding gamma rows wait for the corner warp)
         if (active && sgptr[s] < sgptr[s + 1]) {
             mbar_wait(x1full + (it & 1), (it >> 1) & 1);
@@ -610,6 +644,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                         for (int q = 0; q < NV; ++q) v[j][q] = fma(-gv, x1[q * k + dc], v[j][q]);
             }
         }
+        SB_TR(2);
         // ---------- local forward sweep, publish end state
         C st[K][NV];
         fwd_local<C, K, L, NV, true>(v, fL, ms, st);
@@ -618,7 +653,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             for (int q = 0; q < NV; ++q)
 #pragma unroll
                 for (int j = 0; j < K; ++j) sfend[(s * R + r0 + q) * K + j] = st[j][q];
+        SB_TR(3);
         named_bar(1, nthr_c);  // B2
+        SB_TR(4);
         // ---------- forward carry (true y at rows a-1..a-K) + correction chain
         if (active && s > 0) {
             C cin[K][NV];
@@ -651,7 +688,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             for (int q = 0; q < NV; ++q)
 #pragma unroll
                 for (int j = 0; j < K; ++j) sbbeg[(s * R + r0 + q) * K + j] = st[j][q];
+        SB_TR(5);
         named_bar(1, nthr_c);  // B3
+        SB_TR(6);
         // ---------- backward carry (true x at rows a+L..a+L+K-1) + correction chain
         // TMA path, band K >= 2: every row is stored from inside the chain as soon as
         // it is final (the last segment runs the chain with zero carries, so there is
@@ -710,6 +749,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                         if (q < nlive && a + i < nQ) __stcs(dst + (int64_t)i * ps + q * p.bstride, (T)v[i][q]);
             }
         }
+        SB_TR(7);
         if (LOADER == LOAD_DIRECT) {  // tile done: lets the corner warp move to tile it+1
             __syncwarp();
             if (lane == 0) mbar_arrive(empty + 0);

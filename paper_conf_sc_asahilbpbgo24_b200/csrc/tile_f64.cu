@@ -13,3 +13,9 @@ int launch_tile_f64(int R, int loader, int K, const KParams &kp, const CUtensorM
     return 5;
 }
 }  // namespace sb
+
+#ifdef SB_TRACE
+extern "C" int sb_trace_dump(long long *host, size_t bytes) {
+    return (int)cudaMemcpyFromSymbol(host, sb::g_sb_trace, bytes);
+}
+#endif
