@@ -20,5 +20,26 @@ for p, npts, bc, mesh, B, layout in cases:
     for dt in (np.float64, np.float32):
         t = torch.from_numpy((b if layout == "batch" else np.ascontiguousarray(b.T)).astype(dt)).cuda()
         sb.solve_(t)
+# advection (uniform stencil and non-uniform BSPLVB), both layouts
+for mesh in ("uniform", "sin"):
+    sb = SplineBuilder(3, 1024, PERIODIC, inputs.breakpoints(1024, mesh))
+    b = inputs.rhs(sb.n, 45, seed=5)
+    sh = torch.linspace(-0.3, 0.7, 45, dtype=torch.float64).cuda()
+    for dt in (np.float64, np.float32):
+        sb.advect_(torch.from_numpy(np.ascontiguousarray(b.T).astype(dt)).cuda(), sh)
+        sb.advect_(torch.from_numpy(b.astype(dt)).cuda(), sh)
+# slabs (3-D TMA) and the 2-D tensor-product builder (warp pass + slab pass)
+sb = SplineBuilder(5, 200, GREVILLE, inputs.breakpoints(inputs.n_cells(5, 200, GREVILLE), "sin"))
+f = torch.from_numpy(np.random.default_rng(1).uniform(-1, 1, (3, sb.n, 40))).cuda()
+sb.solve_slabs_(f, 40, 40, 3, sb.n * 40)
+h1 = SplineBuilder(3, 128, PERIODIC)
+h2 = SplineBuilder(5, 96, GREVILLE, inputs.breakpoints(inputs.n_cells(5, 96, GREVILLE), "sin"))
+from paper_conf_sc_asahilbpbgo24_b200 import solve_2d_  # noqa: E402
+solve_2d_(h1, h2, torch.from_numpy(np.random.default_rng(2).uniform(-1, 1, (5, h2.n, h1.n))).cuda())
+# mixed boundary conditions (Hermite at one end, Greville at the other)
+from paper_conf_sc_asahilbpbgo24_b200 import bc_mixed  # noqa: E402
+bcm = bc_mixed(HERMITE, GREVILLE)
+sb = SplineBuilder(5, 300, bcm, inputs.breakpoints(inputs.n_cells(5, 300, bcm), "sin"))
+sb.solve_(torch.from_numpy(np.random.default_rng(3).uniform(-1, 1, (sb.n, 50))).cuda())
 torch.cuda.synchronize()
 print("sanitize run done")
