@@ -824,6 +824,8 @@ __device__ __forceinline__ C nu_value(double x, int c, const double *xe, const C
         double saved = 0.0;
 #pragma unroll
         for (int r = 0; r <= j; ++r) {
+            // (computing the reciprocals with __drcp_rn instead of loading them,
+            // -48 B of shared traffic per point, measured 1.32 vs 1.02 ms for ADVNU)
             const double term = b[r] * rk[(r - j) * RS + j];  // 1/(t_{c+1+r} - t_{c-j+r})
             b[r] = fma(tk[1 + r] - x, term, saved);
             saved = (x - tk[r - j]) * term;

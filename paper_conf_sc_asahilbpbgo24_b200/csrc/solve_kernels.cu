@@ -184,6 +184,25 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
         return 0;
     };
 
+    static const int small_env = [] {  // SB_SMALL_KERNEL=1 serial / 2 warp / 3 tile kernel for batch-contiguous (A/B)
+        const char *e = getenv("SB_SMALL_KERNEL");
+        return e ? atoi(e) : 0;
+    }();
+    // tiny problems (C1: 16 x 8) are launch/latency-bound: the warp kernel's lighter
+    // prologue wins (C1 graph-timed: warp 5.4 us, serial 6.4 us, tile 7.3 us)
+    const bool tiny = a.nslab == 1 && P.n <= 64 && a.batch <= 64 && P.seg[2].S > 0;
+    if ((small_env == 2 || (small_env == 0 && tiny)) && a.nslab == 1)
+        return launch_warp(P, a, num_sms, max_smem, err, errlen);
+    if (small_env == 1 && a.nslab == 1) {
+        KParams kp{};
+        kp.P = P;
+        kp.rhs = a.rhs;
+        kp.batch = a.batch;
+        kp.bstride = a.bstride;
+        kp.pstride = a.pstride;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
+        return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
+    }
     const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
     const int L = G.L;
     KParams kp{};
