@@ -191,6 +191,49 @@ def test_c3_full_size_sampled(torch_cuda, bc, npts):
     assert o.residual(got[:, idx], b[:, idx]) <= TOL64
 
 
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_c4_full_size_sampled(torch_cuda, dtype):
+    """C4 at full size in the bench's configuration: n = 1024, 64*64*32 =
+    131072 right-hand sides, x contiguous (point layout: the warp kernel's
+    bulk-copy pipeline), on a seeded sample of RHS incl. first/last; fp32
+    against the oracle run on the fp32-rounded inputs."""
+    torch = torch_cuda
+    sb, o = make(3, 1024, PERIODIC, "uniform")
+    B = 64 * 64 * 32
+    host = np.ascontiguousarray(inputs.rhs(sb.n, B, seed=1234).T.astype(np.float64 if dtype == "f64" else np.float32))
+    t = torch.from_numpy(host).cuda()
+    sb.solve_(t)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    idx = np.unique(np.concatenate([[0, B - 1], np.random.default_rng(5).choice(B, 1024, replace=False)]))
+    b_s = np.ascontiguousarray(host[idx].T.astype(np.float64))
+    ref = o.solve(b_s)
+    x = np.ascontiguousarray(got[idx].T.astype(np.float64))
+    assert rel_coef_error(x, ref) <= (TOL64 if dtype == "f64" else TOL32)
+    if dtype == "f64":
+        assert o.residual(x, b_s) <= TOL64
+
+
+@pytest.mark.parametrize("kind", ["uniform", "sin"])
+def test_advect_full_size_sampled(torch_cuda, kind):
+    """The advection workloads at full size (Nx = 1024, Nv = 1e5, x
+    contiguous, |shift| <= 2.5 cells as in bench.py), sampled rows against
+    the oracle's solve + evaluation at the feet (Algorithm 2)."""
+    torch = torch_cuda
+    sb, o = make(3, 1024, PERIODIC, kind)
+    B = 100000
+    b = inputs.rhs(sb.n, B, seed=1234)
+    v = -1.0 + 2.0 * np.arange(B, dtype=np.float64) / B
+    shift = v * (2.5 / o.N)
+    t = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()
+    sb.advect_(t, torch.from_numpy(shift).cuda())
+    torch.cuda.synchronize()
+    got = t.cpu().numpy()
+    idx = np.unique(np.concatenate([[0, B - 1], np.random.default_rng(6).choice(B, 1024, replace=False)]))
+    ref = o.advect(np.ascontiguousarray(b[:, idx]), shift[idx])
+    assert rel_coef_error(np.ascontiguousarray(got[idx].T), ref) <= TOL64
+
+
 def test_c5_shards_bitwise_equal_and_sampled_parity(torch_cuda):
     """C5 recipe: device-generated RHS (inputs.rhs_device), sharded into
     contiguous slices; each shard solved on its own equals the unsharded solve
