@@ -328,6 +328,45 @@ __device__ __forceinline__ void getrs_small(C *x1, const C *lu, const int *piv, 
     }
 }
 
+// x1 <- delta'^{-1} x1 with x1 in registers (warp kernel corner, k <= KR;
+// unrolled and guarded by d < k, no dynamic register indexing; the same
+// operations in the same order as getrs_small; LAPACK pivots, piv[d] >= d).
+// Measured (A/B against the lane-0 corner, two sessions): C4 0.383 -> 0.352
+// ms, C6 0.389 -> 0.379 ms, C6NU 0.591 -> 0.618 ms (pass 1 has k = 2).
+// Restricting it to k == 1, or instantiating 1 slot, changes the code
+// generation of the whole kernel and loses the C4 gain (0.374 ms).
+constexpr int WCORNER_KREG = 8;
+template <typename C, int KR>
+__device__ __forceinline__ void wgetrs_reg(C (&x)[KR], const C *lu, const int *piv, int k) {
+#pragma unroll
+    for (int d = 0; d < KR; ++d) {
+        if (d < k) {
+            const int pv = piv[d];
+            C xp = x[d];
+#pragma unroll
+            for (int j = d + 1; j < KR; ++j) xp = j == pv ? x[j] : xp;
+            const C t = x[d];
+            x[d] = xp;
+#pragma unroll
+            for (int j = d + 1; j < KR; ++j) x[j] = j == pv ? t : x[j];
+        }
+    }
+#pragma unroll
+    for (int i = 1; i < KR; ++i)
+        if (i < k)
+#pragma unroll
+            for (int j = 0; j < i; ++j) x[i] = fma(-lu[i * k + j], x[j], x[i]);
+#pragma unroll
+    for (int i = KR - 1; i >= 0; --i)
+        if (i < k) {
+            C acc = x[i];
+#pragma unroll
+            for (int j = i + 1; j < KR; ++j)
+                if (j < k) acc = fma(-lu[i * k + j], x[j], acc);
+            x[i] = acc / lu[i * k + i];
+        }
+}
+
 // Stage the constants of one segment plan + the corner data (+ the advection
 // geometry) into shared memory with bulk async copies (cp.async.bulk, one
 // instruction per array, completion on one mbarrier) instead of a
@@ -1016,7 +1055,45 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
             __syncwarp();
         }
         // ---------- corner: x1 = delta'^{-1} (s1*b1 - Lambda b0), then b0 -= gamma x1
-        if (k > 0) {
+        // fp64 solve: x1 in registers on every lane (the xor reduction leaves the
+        // sum on all lanes), getrs on registers, then gamma row by row on parallel
+        // lanes -- no serial chain of dependent shared-memory round trips on lane 0
+        // (measured: C4 fp64 0.383 -> 0.352 ms, C6 0.389 -> 0.379 ms; the same code
+        // made the fp32 solve and the advection step slower, 0.182 -> 0.211 and
+        // 0.385 -> 0.460 ms, so they keep the lane-0 corner)
+        constexpr bool REG_CORNER = sizeof(T) == 8 && !ADV;
+        if (REG_CORNER && k > 0 && k <= WCORNER_KREG) {
+            C xr[WCORNER_KREG];
+#pragma unroll
+            for (int d = 0; d < WCORNER_KREG; ++d) {
+                C acc = C(0);
+                if (d < k) {
+                    acc = lane == 0 ? rowbuf[sdrow[d]] * sdscale[d] : C(0);
+                    for (int e = slamptr[d] + lane; e < slamptr[d + 1]; e += 32)
+                        acc = fma(-slamv[e], rowbuf[s_lo + slamc[e]], acc);
+#pragma unroll
+                    for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+                }
+                xr[d] = acc;
+            }
+            wgetrs_reg<C, WCORNER_KREG>(xr, sdlu, sdpiv, k);
+            auto xsel = [&](int c) {
+                C r = xr[0];
+#pragma unroll
+                for (int j = 1; j < WCORNER_KREG; ++j) r = j == c ? xr[j] : r;
+                return r;
+            };
+            __syncwarp();  // every lane has read its Lambda columns and delta rows of the row buffer
+            for (int e = lane; e < P.gam_nnz; e += 32) {
+                const int row = sgamr[e];
+                if (e > 0 && sgamr[e - 1] == row) continue;  // the lane of the row's first entry does the row
+                C val = rowbuf[s_lo + row];
+                for (int f = e; f < P.gam_nnz && sgamr[f] == row; ++f) val -= sgamv[f] * xsel(sgamc[f]);
+                rowbuf[s_lo + row] = val;
+            }
+            if (lane < k) rowbuf[sdrow[lane]] = xsel(lane);
+            __syncwarp();
+        } else if (k > 0) {
             for (int d = 0; d < k; ++d) {
                 C acc = lane == 0 ? rowbuf[sdrow[d]] * sdscale[d] : C(0);
                 for (int e = slamptr[d] + lane; e < slamptr[d + 1]; e += 32)
