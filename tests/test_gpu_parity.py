@@ -107,6 +107,31 @@ def test_parity_point_contiguous(torch_cuda, n_points, dtype):
     assert rel_coef_error(got, ref) <= (TOL64 if dtype == np.float64 else TOL32)
 
 
+@pytest.mark.parametrize("case", [(5, 1000, GREVILLE, "sin"), (5, 996, HERMITE, "sin"), (5, 1000, PERIODIC, "jitter"),
+                                  (4, 1000, PERIODIC, "uniform"), (3, 200, GREVILLE | (HERMITE << 4), "jitter"),
+                                  (2, 40, GREVILLE, "sin")],
+                         ids=lambda c: f"p{c[0]}-n{c[1]}-bc{c[2]}-{c[3]}")
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_parity_point_contiguous_corners(torch_cuda, case, dtype):
+    """Point layout (warp kernel) for delta orders k = 2..6 and mixed ends:
+    the fp64 corner runs on registers of every lane (getrs + gamma rows on
+    parallel lanes), the fp32 one on lane 0."""
+    torch = torch_cuda
+    p, npts, bc, kind = case
+    sb, o = make(p, npts, bc, kind)
+    B = 333
+    b = inputs.rhs(sb.n, B, seed=808, degree=p, bc=bc).astype(dtype)
+    t = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()
+    sb.solve_(t)
+    torch.cuda.synchronize()
+    got = t.cpu().numpy().T.astype(np.float64)
+    b64 = b.astype(np.float64)
+    ref = o.solve(b64)
+    assert rel_coef_error(got, ref) <= (TOL64 if dtype == np.float64 else TOL32), sb.info()["k"]
+    if dtype == np.float64:
+        assert o.residual(got, b64) <= TOL64
+
+
 def test_strided_matches_contiguous(torch_cuda):
     """The same RHS in batch-contiguous (tile kernel) and point-contiguous
     (warp kernel) layouts agree to rounding.  The two kernels use different
