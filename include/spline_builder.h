@@ -94,6 +94,18 @@ spline_builder_t spline_builder_create(int degree, int n_points, int bc, const d
 spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, const double *knots,
                                           int split_lo, int split_hi, int flags);
 
+/* spline_builder_update -- new mesh, same handle (SURVEY 8(f)4 "matrices
+ * that change"; the factorisation is done once per mesh on the host and
+ * copied to the device).  Rebuilds the collocation matrix, the Schur
+ * split of Eq. 3 and every factor for the breakpoints `knots` (host
+ * pointer, N+1 values, same meaning as in create; NULL = uniform), keeping
+ * the create-time degree, n_points, bc and split request.  The device
+ * constants are replaced synchronously; the caller ensures no solve on h is
+ * in flight (as for destroy).  On any error (bad knots, singular factor,
+ * out of memory) the handle keeps its previous mesh and factors and the
+ * status code is returned. */
+int spline_builder_update(spline_builder_t h, const double *knots);
+
 /*
  * spline_builder_solve -- in-place batched solve of fp64 right-hand sides
  * (Algorithm 1; fused kernel of Listing 6).

@@ -82,6 +82,20 @@ class SplineBuilder:
     def __exit__(self, *exc):
         self.close()
 
+    def update(self, knots=None):
+        """New breakpoints for the same degree / n_points / bc / split request
+        (``spline_builder_update``): the factors are rebuilt and replaced in
+        the handle.  Synchronise streams that use this handle first.  On
+        error the handle keeps its previous mesh."""
+        kbuf = None
+        if knots is not None:
+            import numpy as np
+            kn = np.ascontiguousarray(knots, dtype=np.float64)
+            kbuf = ctypes.c_void_p(kn.ctypes.data)
+        _lib.check(self._lib.spline_builder_update(self._h, kbuf))
+        if knots is not None:
+            self._knots = kn
+
     # ------------------------------------------------------------- queries
     def info(self) -> dict:
         inf = SplineBuilderInfo()

@@ -19,7 +19,7 @@ SB_FLAG_HOST_ONLY = 1
 
 # every symbol include/spline_builder.h declares (checked by tests/test_abi.py)
 EXPORTS = [
-    "spline_builder_create", "spline_builder_create_ex", "spline_builder_solve", "spline_builder_solve_f32",
+    "spline_builder_create", "spline_builder_create_ex", "spline_builder_update", "spline_builder_solve", "spline_builder_solve_f32",
     "spline_builder_solve_strided", "spline_builder_solve_slabs", "spline_builder_solve_2d", "spline_builder_advect", "spline_builder_solve_host", "spline_builder_destroy",
     "spline_builder_get_info", "spline_builder_nbasis", "spline_builder_get_blocks",
     "spline_builder_solve_cpu_plan", "spline_builder_last_error", "spline_builder_last_status",
@@ -73,6 +73,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.spline_builder_advect.argtypes = [vp, dp, i32, i64, i64, i64, dp, vp]
     lib.spline_builder_solve_host.restype = i32
     lib.spline_builder_solve_host.argtypes = [vp, dp, i32, i64, i64]
+    lib.spline_builder_update.restype = i32
+    lib.spline_builder_update.argtypes = [vp, dp]
     lib.spline_builder_destroy.restype = None
     lib.spline_builder_destroy.argtypes = [vp]
     lib.spline_builder_get_info.restype = i32

@@ -36,6 +36,7 @@ struct spline_builder {
     int device = -1;
     int num_sms = 0;
     bool host_only = false;
+    int c_degree = 0, c_npoints = 0, c_bc = 0, c_split_lo = -1, c_split_hi = -1;  // create arguments (update)
     void *blob = nullptr;  // device constants
     size_t blob_bytes = 0;
     sb::DevPlan dp{};
@@ -252,12 +253,48 @@ spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, cons
         fail(SB_INVALID_ARG, "unexpected failure in create"); delete h; return nullptr;
     }
     h->host_only = (flags & SB_FLAG_HOST_ONLY) != 0;
+    h->c_degree = degree; h->c_npoints = n_points; h->c_bc = bc; h->c_split_lo = split_lo; h->c_split_hi = split_hi;
     if (!h->host_only) {
         if (cudaGetDevice(&h->device) != cudaSuccess) { fail(SB_CUDA, "no CUDA device"); delete h; return nullptr; }
         cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device);
         if (upload(h)) { spline_builder_destroy(h); return nullptr; }
     }
     return h;
+}
+
+int spline_builder_update(spline_builder_t h, const double *knots) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    sb::Plan fresh;
+    try {
+        sb::Status st = sb::build_plan(fresh, h->c_degree, h->c_npoints, h->c_bc, knots, h->c_split_lo, h->c_split_hi);
+        if (st.code) return fail(st.code, st.msg);
+    } catch (const std::bad_alloc &) {
+        return fail(SB_NOMEM, "out of host memory in update");
+    } catch (...) {
+        return fail(SB_INVALID_ARG, "unexpected failure in update");
+    }
+    if (h->host_only) { h->plan = std::move(fresh); return SB_OK; }
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != h->device) cudaSetDevice(h->device);
+    // keep the old state until the new blob is on the device; restore it on failure
+    sb::Plan old_plan = std::move(h->plan);
+    void *old_blob = h->blob;
+    size_t old_bytes = h->blob_bytes;
+    sb::DevPlan old_dp = h->dp;
+    h->plan = std::move(fresh);
+    h->blob = nullptr;
+    int rc = upload(h);  // synchronous cudaMemcpy: the new constants are in place on return
+    if (rc) {
+        if (h->blob) cudaFree(h->blob);
+        h->plan = std::move(old_plan); h->blob = old_blob; h->blob_bytes = old_bytes; h->dp = old_dp;
+        const std::string msg = g_err;
+        if (cur != h->device) cudaSetDevice(cur);
+        return fail(rc, msg);
+    }
+    if (old_blob) cudaFree(old_blob);  // the caller guaranteed no solve on h is in flight
+    if (cur != h->device) cudaSetDevice(cur);
+    return SB_OK;
 }
 
 spline_builder_t spline_builder_create(int degree, int n_points, int bc, const double *knots) {

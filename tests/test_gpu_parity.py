@@ -485,3 +485,37 @@ def test_2d_full_size_chunked_sampled(torch_cuda):
     A1, A2 = o1.matrix(), o2.matrix()
     res = np.abs(A2 @ out[3] @ A1.T - F[3]).max() / np.abs(F[3]).max()
     assert res <= 1e-12
+
+
+@pytest.mark.parametrize("p,npts,bc", [(3, 1000, PERIODIC), (5, 1000, GREVILLE), (5, 996, HERMITE),
+                                       (4, 1024, PERIODIC)])
+def test_update_new_mesh_parity(torch_cuda, p, npts, bc):
+    """NEXT f4 (matrices that change): spline_builder_update moves a device
+    handle to a new mesh; batch-contiguous solves, point-contiguous solves and
+    (periodic) the advection step then match the oracle on the new mesh and
+    a handle created on it bit for bit."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder
+    N = inputs.n_cells(p, npts, bc)
+    sb = SplineBuilder(p, npts, bc, inputs.breakpoints(N, "uniform"))
+    b = inputs.rhs(sb.n, 333, seed=17, degree=p, bc=bc)
+    gpu_solve(torch, sb, b.copy())
+    for kind, seed in (("sin", 42), ("jitter", 3), ("uniform", 42)):
+        x = inputs.breakpoints(N, kind, seed=seed)
+        sb.update(x)
+        o = Oracle(p, npts, bc, x)
+        fresh = SplineBuilder(p, npts, bc, x)
+        got = gpu_solve(torch, sb, b.copy())
+        assert rel_coef_error(got, o.solve(b)) <= TOL64
+        assert np.array_equal(got, gpu_solve(torch, fresh, b.copy()))
+        t = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()
+        sb.solve_(t)
+        torch.cuda.synchronize()
+        assert rel_coef_error(t.cpu().numpy().T, o.solve(b)) <= TOL64
+        if bc == PERIODIC:
+            shift = np.linspace(-2.5, 2.5, b.shape[1]) / N
+            t = torch.from_numpy(b.copy()).cuda()
+            sb.advect_(t, torch.from_numpy(shift).cuda())
+            torch.cuda.synchronize()
+            assert rel_coef_error(t.cpu().numpy(), o.advect(b, shift)) <= TOL64
+        fresh.close()

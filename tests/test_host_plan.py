@@ -172,3 +172,43 @@ def test_mixed_bc_host_plan_matches_oracle(case):
     o = Oracle(p, npts, bc, x)
     b = inputs.rhs(o.n, 9, seed=3, degree=p, bc=bc)
     assert rel_coef_error(sb.solve_cpu_plan_(b.copy()), o.solve(b)) < 1e-13
+
+
+UPDATE = [(3, 1000, PERIODIC), (4, 200, PERIODIC), (5, 1000, GREVILLE), (5, 996, HERMITE),
+          (3, 60 + 3 - 1, inputs.bc_mixed(HERMITE, GREVILLE))]
+
+
+@pytest.mark.parametrize("case", UPDATE, ids=[f"p{c[0]}-n{c[1]}-bc{c[2]}" for c in UPDATE])
+def test_update_new_mesh_matches_oracle(case):
+    """spline_builder_update (NEXT row f4, matrices that change): a handle
+    moved from one mesh to another solves like the oracle on the new mesh and
+    carries the same factors as a handle created on it."""
+    p, npts, bc = case
+    sb, _ = host(p, npts, bc, "uniform")
+    N = inputs.n_cells(p, npts, bc)
+    for kind, seed in (("sin", 42), ("jitter", 7), ("uniform", 42)):
+        x = inputs.breakpoints(N, kind, seed=seed)
+        sb.update(x)
+        fresh = SplineBuilder(p, npts, bc, x, host_only=True)
+        assert sb.info() == fresh.info()
+        o = Oracle(p, npts, bc, x)
+        b = inputs.rhs(o.n, 7, seed=5, degree=p, bc=bc)
+        got = sb.solve_cpu_plan_(b.copy())
+        assert rel_coef_error(got, o.solve(b)) < 1e-13
+        assert np.array_equal(got, fresh.solve_cpu_plan_(b.copy()))
+
+
+def test_update_failure_keeps_previous_mesh():
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilderError
+    p, npts = 3, 100
+    x = inputs.breakpoints(npts, "sin")
+    sb = SplineBuilder(p, npts, PERIODIC, x, host_only=True)
+    o = Oracle(p, npts, PERIODIC, x)
+    b = inputs.rhs(o.n, 3, seed=9, degree=p)
+    want = sb.solve_cpu_plan_(b.copy())
+    bad = x.copy()
+    bad[10] = bad[12]                                  # not strictly increasing
+    with pytest.raises(SplineBuilderError):
+        sb.update(bad)
+    assert np.array_equal(sb.solve_cpu_plan_(b.copy()), want)
+    assert rel_coef_error(want, o.solve(b)) < 1e-13
