@@ -41,5 +41,12 @@ from paper_conf_sc_asahilbpbgo24_b200 import bc_mixed  # noqa: E402
 bcm = bc_mixed(HERMITE, GREVILLE)
 sb = SplineBuilder(5, 300, bcm, inputs.breakpoints(inputs.n_cells(5, 300, bcm), "sin"))
 sb.solve_(torch.from_numpy(np.random.default_rng(3).uniform(-1, 1, (sb.n, 50))).cuda())
+# spline_builder_update: a handle moved to a new mesh, then solved and advected
+sb = SplineBuilder(3, 1000, PERIODIC)
+for mesh in ("sin", "jitter"):
+    sb.update(inputs.breakpoints(1000, mesh))
+    b = inputs.rhs(sb.n, 65, seed=7)
+    sb.solve_(torch.from_numpy(b).cuda())
+    sb.advect_(torch.from_numpy(b).cuda(), torch.linspace(-0.3, 0.7, 65, dtype=torch.float64).cuda())
 torch.cuda.synchronize()
 print("sanitize run done")
