@@ -28,7 +28,7 @@
 extern "C" {
 #endif
 
-typedef struct spline_builder *spline_builder_t; /* opaque, immutable after create */
+typedef struct spline_builder *spline_builder_t; /* opaque; changed only by spline_builder_update */
 
 /* boundary conditions (PAPER.md P:55 periodic; non-periodic per BASELINE C3) */
 enum { SB_PERIODIC = 0, SB_GREVILLE = 1, SB_HERMITE = 2 };
@@ -103,7 +103,12 @@ spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, cons
  * constants are replaced synchronously; the caller ensures no solve on h is
  * in flight (as for destroy).  On any error (bad knots, singular factor,
  * out of memory) the handle keeps its previous mesh and factors and the
- * status code is returned. */
+ * status code is returned.
+ * CUDA graphs: a solve captured before the update keeps the OLD mesh's
+ * constants (its launch arguments point into the previous device blob, which
+ * stays allocated until destroy, so replay is memory-safe but uses the old
+ * matrix).  Re-capture graphs after an update to solve with the new mesh.
+ * Each host update retires one blob (~10-200 KB) until destroy. */
 int spline_builder_update(spline_builder_t h, const double *knots);
 
 /*
@@ -231,6 +236,11 @@ int spline_builder_solve_cpu_plan(spline_builder_t h, double *rhs, int64_t batch
                                   int64_t point_stride);
 
 const char *spline_builder_last_error(void); /* thread-local; never NULL */
+/* Kernel the last solve call on the calling thread launched, with its
+ * configuration, e.g. "tile<f64,K=1,R=16,TMA>" (batch-contiguous tile kernel
+ * fed by TMA), "warp<f64,K=1,L=33,BULK>", "serial<f64,K=3>"; "" before the
+ * first solve.  Thread-local, never NULL; for tests and diagnostics. */
+const char *spline_builder_last_kernel(void);
 int spline_builder_last_status(void);        /* status of the last failed call */
 const char *spline_builder_version(void);
 

@@ -22,7 +22,42 @@ def bc_mixed(lo: int, hi: int) -> int:
     """SB_BC(lo, hi) of include/spline_builder.h: different conditions at x_0 / x_N."""
     return lo if lo == hi else lo | (hi << 4)
 
-__all__ = ["SplineBuilder", "SplineBuilderError", "PERIODIC", "GREVILLE", "HERMITE", "load_library", "solve_2d_", "bc_mixed"]
+last_kernel = _lib.last_kernel
+
+__all__ = ["last_kernel", "SplineBuilder", "SplineBuilderError", "PERIODIC", "GREVILLE", "HERMITE", "load_library", "solve_2d_", "bc_mixed"]
+
+
+def n_cells_of(degree: int, n_points: int, bc: int) -> int:
+    """Number of cells N (so N+1 breakpoints) fixed by (degree, n_points, bc),
+    as stated for spline_builder_create in include/spline_builder.h."""
+    p = int(degree)
+    nbc = (p - 1) // 2 if p % 2 else p // 2
+    if bc == PERIODIC:
+        return int(n_points)
+    if bc == GREVILLE:
+        return int(n_points) - p
+    if bc == HERMITE:
+        return int(n_points) - 1 if p % 2 else int(n_points)
+    lo, hi = bc & 15, (bc >> 4) & 15
+    return int(n_points) - p + (nbc if lo == HERMITE else 0) + (nbc if hi == HERMITE else 0)
+
+
+def _knots_arg(knots, n_cells: int):
+    """Contiguous fp64 copy of the breakpoints, checked to hold N+1 values
+    (the C side reads exactly that many)."""
+    import numpy as np
+    kn = np.ascontiguousarray(knots, dtype=np.float64)
+    if kn.ndim != 1 or kn.shape[0] != n_cells + 1:
+        raise ValueError(f"knots must be a 1-D array of N+1 = {n_cells + 1} breakpoints, got shape {kn.shape}")
+    return kn
+
+
+def _check_extent(t, last_index: int, what: str = "rhs"):
+    """The C side addresses elements [0, last_index] from t.data_ptr(): they
+    must lie inside t's storage."""
+    avail = (t.untyped_storage().nbytes() - t.storage_offset() * t.element_size()) // t.element_size()
+    if last_index >= avail:
+        raise ValueError(f"{what}: strides address element {last_index} but only {avail} are allocated")
 
 
 def load_library():
@@ -52,8 +87,7 @@ class SplineBuilder:
         self._lib = lib
         kbuf = None
         if knots is not None:
-            import numpy as np
-            self._knots = np.ascontiguousarray(knots, dtype=np.float64)
+            self._knots = _knots_arg(knots, n_cells_of(degree, n_points, bc))
             kbuf = ctypes.c_void_p(self._knots.ctypes.data)
         lo, hi = (-1, -1) if split is None else split
         flags = SB_FLAG_HOST_ONLY if host_only else 0
@@ -89,8 +123,7 @@ class SplineBuilder:
         error the handle keeps its previous mesh."""
         kbuf = None
         if knots is not None:
-            import numpy as np
-            kn = np.ascontiguousarray(knots, dtype=np.float64)
+            kn = _knots_arg(knots, self.info()["n_cells"])
             kbuf = ctypes.c_void_p(kn.ctypes.data)
         _lib.check(self._lib.spline_builder_update(self._h, kbuf))
         if knots is not None:
@@ -134,14 +167,28 @@ class SplineBuilder:
             else:
                 raise ValueError(f"no dimension of size n={self.n}")
         else:
-            bs = batch_stride
-            batch = rhs.shape[1] if bs == 1 else rhs.shape[0]
+            bs = int(batch_stride)
+            if bs == 1:
+                if rhs.shape[0] != self.n:
+                    raise ValueError(f"batch_stride=1 needs shape (n={self.n}, batch), got {tuple(rhs.shape)}")
+                batch = rhs.shape[1]
+            else:
+                if bs != rhs.shape[1] or rhs.shape[1] < self.n:
+                    raise ValueError(f"batch_stride={bs} needs shape (batch, {bs}) with {bs} >= n={self.n}, "
+                                     f"got {tuple(rhs.shape)}")
+                batch = rhs.shape[0]
         fn = self._lib.spline_builder_solve if rhs.dtype == torch.float64 else self._lib.spline_builder_solve_f32
         _lib.check(fn(self._h, ctypes.c_void_p(rhs.data_ptr()), int(batch), int(bs), _stream_handle(stream)))
         return rhs
 
     def solve_strided_(self, rhs, batch: int, batch_stride: int, point_stride: int, stream=None):
         import torch
+        if not rhs.is_cuda:
+            raise ValueError("rhs must be a CUDA tensor")
+        if rhs.dtype not in (torch.float64, torch.float32):
+            raise TypeError("rhs must be float64 or float32")
+        if batch > 0:
+            _check_extent(rhs, (batch - 1) * batch_stride + (self.n - 1) * point_stride)
         dt = SB_F64 if rhs.dtype == torch.float64 else SB_F32
         _lib.check(self._lib.spline_builder_solve_strided(self._h, ctypes.c_void_p(rhs.data_ptr()), dt, int(batch),
                                                           int(batch_stride), int(point_stride),
@@ -154,6 +201,10 @@ class SplineBuilder:
         import torch
         if not rhs.is_cuda:
             raise ValueError("rhs must be a CUDA tensor")
+        if rhs.dtype not in (torch.float64, torch.float32):
+            raise TypeError("rhs must be float64 or float32")
+        if batch > 0 and nslab > 0:
+            _check_extent(rhs, (nslab - 1) * slab_stride + (self.n - 1) * ld + batch - 1)
         dt = SB_F64 if rhs.dtype == torch.float64 else SB_F32
         _lib.check(self._lib.spline_builder_solve_slabs(self._h, ctypes.c_void_p(rhs.data_ptr()), dt, int(batch),
                                                         int(ld), int(nslab), int(slab_stride),
@@ -180,7 +231,11 @@ class SplineBuilder:
             else:
                 raise ValueError(f"no dimension of size n={self.n}")
         else:
-            bs = batch_stride
+            bs = int(batch_stride)
+            if bs == 1 and f.shape[0] != self.n:
+                raise ValueError(f"batch_stride=1 needs shape (n={self.n}, batch), got {tuple(f.shape)}")
+            if bs != 1 and (bs != f.shape[1] or bs < self.n):
+                raise ValueError(f"batch_stride={bs} needs shape (batch, {bs}) with {bs} >= n={self.n}")
             batch, pst = (f.shape[1], f.shape[1]) if bs == 1 else (f.shape[0], 1)
         if shift.numel() != batch:
             raise ValueError("shift must have one entry per right-hand side")
@@ -199,12 +254,28 @@ class SplineBuilder:
         except ImportError:  # pragma: no cover
             is_t = False
         if is_t:
+            if arr.is_cuda:
+                raise ValueError("solve_host_ takes host memory (use solve_ for CUDA tensors)")
+            if arr.dtype not in (torch.float64, torch.float32):
+                raise TypeError("host array must be float64 or float32")
+            if arr.dim() != 2 or arr.stride(1) != 1:
+                raise ValueError("host array must be 2-D (n, batch) with unit inner stride")
             dt = SB_F64 if arr.dtype == torch.float64 else SB_F32
             ptr, batch, ld0 = arr.data_ptr(), arr.shape[1], arr.stride(0)
         else:
             import numpy as np
+            if arr.dtype not in (np.float64, np.float32):
+                raise TypeError("host array must be float64 or float32")
+            if arr.ndim != 2 or arr.strides[1] != arr.itemsize or arr.strides[0] % arr.itemsize:
+                raise ValueError("host array must be 2-D (n, batch) with unit inner stride")
+            if not arr.flags.writeable:
+                raise ValueError("host array must be writeable (the solve is in place)")
             dt = SB_F64 if arr.dtype == np.float64 else SB_F32
             ptr, batch, ld0 = arr.ctypes.data, arr.shape[1], arr.strides[0] // arr.itemsize
+        if arr.shape[0] != self.n:
+            raise ValueError(f"host array must have n={self.n} rows, got {arr.shape[0]}")
+        if ld is not None and ld != ld0:
+            raise ValueError(f"ld={ld} differs from the array's row stride {ld0}")
         _lib.check(self._lib.spline_builder_solve_host(self._h, ctypes.c_void_p(ptr), dt, int(batch),
                                                        int(ld if ld is not None else ld0)))
         return arr

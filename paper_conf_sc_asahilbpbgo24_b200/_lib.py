@@ -23,6 +23,7 @@ EXPORTS = [
     "spline_builder_solve_strided", "spline_builder_solve_slabs", "spline_builder_solve_2d", "spline_builder_advect", "spline_builder_solve_host", "spline_builder_destroy",
     "spline_builder_get_info", "spline_builder_nbasis", "spline_builder_get_blocks",
     "spline_builder_solve_cpu_plan", "spline_builder_last_error", "spline_builder_last_status",
+    "spline_builder_last_kernel",
     "spline_builder_version",
 ]
 
@@ -89,6 +90,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.spline_builder_last_error.argtypes = []
     lib.spline_builder_last_status.restype = i32
     lib.spline_builder_last_status.argtypes = []
+    lib.spline_builder_last_kernel.restype = ctypes.c_char_p
+    lib.spline_builder_last_kernel.argtypes = []
     lib.spline_builder_version.restype = ctypes.c_char_p
     lib.spline_builder_version.argtypes = []
     _lib = lib
@@ -97,6 +100,11 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
 
 def last_error() -> str:
     return load().spline_builder_last_error().decode()
+
+
+def last_kernel() -> str:
+    """Kernel (and configuration) of the calling thread's last solve."""
+    return load().spline_builder_last_kernel().decode()
 
 
 def check(status: int) -> None:

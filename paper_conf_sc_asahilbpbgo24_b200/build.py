@@ -1,7 +1,8 @@
 """In-tree build of libsplinebuilder.so (C ABI + sm_100a kernels).
 
-nvcc cross-compiles for sm_100a without a GPU.  The library links the CUDA
-runtime statically and never links torch.
+nvcc cross-compiles for sm_100a without a GPU.  The library links the shared
+CUDA runtime (libcudart.so.12; when torch is loaded first, its copy of the
+runtime is the one used) and never links torch.
 """
 from __future__ import annotations
 
@@ -75,7 +76,8 @@ def build(force: bool = False, verbose: bool = False, extra_flags: tuple = (), l
     with ThreadPoolExecutor(max_workers=max(1, min(len(jobs), os.cpu_count() or 4))) as ex:
         list(ex.map(run, jobs))
     if force or _newer(LIB, objs):
-        cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", LIB + ".tmp", *objs, "-lpthread", "-ldl", "-lrt"]
+        cmd = [NVCC, *ARCH, "-shared", "-cudart", "shared", "-Xlinker", "-rpath=" + os.path.join(CUDA_HOME, "lib64"),
+               "-o", LIB + ".tmp", *objs, "-lpthread", "-ldl", "-lrt"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed: {' '.join(cmd)}\n{r.stdout}\n{r.stderr}")

@@ -39,6 +39,9 @@ struct spline_builder {
     int c_degree = 0, c_npoints = 0, c_bc = 0, c_split_lo = -1, c_split_hi = -1;  // create arguments (update)
     void *blob = nullptr;  // device constants
     size_t blob_bytes = 0;
+    // blobs replaced by update(): kept until destroy, so kernels captured in a
+    // CUDA graph before an update stay memory-safe (they keep the old mesh)
+    std::vector<void *> retired;
     sb::DevPlan dp{};
     // staging for solve_host
     std::mutex host_mu;
@@ -157,6 +160,10 @@ int upload(spline_builder *h) {
     if (e != cudaSuccess) return fail(SB_NOMEM, std::string("cudaMalloc(blob): ") + cudaGetErrorString(e));
     e = cudaMemcpy(h->blob, pk.bytes.data(), pk.bytes.size(), cudaMemcpyHostToDevice);
     if (e != cudaSuccess) return fail(SB_CUDA, std::string("cudaMemcpy(blob): ") + cudaGetErrorString(e));
+    // a copy from pageable memory may still be in flight when cudaMemcpy returns;
+    // solves may be issued on non-blocking streams that do not order against it
+    e = cudaStreamSynchronize(0);
+    if (e != cudaSuccess) return fail(SB_CUDA, std::string("sync after blob upload: ") + cudaGetErrorString(e));
     auto at = [&](size_t off) { return (const void *)((const unsigned char *)h->blob + off); };
     sb::DevPlan &d = h->dp;
     d.n = P.n; d.nQ = nQ; d.s_lo = P.s_lo; d.k = k; d.K = K;
@@ -292,7 +299,7 @@ int spline_builder_update(spline_builder_t h, const double *knots) {
         if (cur != h->device) cudaSetDevice(cur);
         return fail(rc, msg);
     }
-    if (old_blob) cudaFree(old_blob);  // the caller guaranteed no solve on h is in flight
+    if (old_blob) h->retired.push_back(old_blob);  // freed at destroy (graphs may still reference it)
     if (cur != h->device) cudaSetDevice(cur);
     return SB_OK;
 }
@@ -446,6 +453,7 @@ void spline_builder_destroy(spline_builder_t h) {
         cudaGetDevice(&cur);
         if (h->device >= 0 && cur != h->device) cudaSetDevice(h->device);
         if (h->blob) cudaFree(h->blob);
+        for (void *b : h->retired) cudaFree(b);
         for (int i = 0; i < 3; ++i) {
             if (h->stage[i]) cudaFree(h->stage[i]);
             if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
@@ -500,6 +508,7 @@ int spline_builder_solve_cpu_plan(spline_builder_t h, double *rhs, int64_t batch
 }
 
 const char *spline_builder_last_error(void) { return g_err.c_str(); }
+const char *spline_builder_last_kernel(void) { return sb::last_kernel(); }
 int spline_builder_last_status(void) { return g_status; }
 const char *spline_builder_version(void) { return "b200-spline-build 0.1 (sm_100a)"; }
 

@@ -56,6 +56,9 @@ struct SolveArgs {
     int64_t slab_stride = 0;
 };
 
+// name + configuration of the kernel the last launch_solve on this thread chose
+const char *last_kernel();
+
 // returns 0 on success, else an SB_* status; fills err on failure
 int launch_solve(const DevPlan &P, const SolveArgs &a, int num_sms, char *err, int errlen);
 

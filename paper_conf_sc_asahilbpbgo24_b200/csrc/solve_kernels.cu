@@ -1,28 +1,45 @@
 // solve_kernels.cu -- host-side dispatch of the fused kernels (kernels.cuh):
 // layout / tile-width / loader choice, shared-memory layout, TMA descriptor.
+#include <atomic>
 #include <cstdlib>
 
 #include "kernels.cuh"
 
 namespace sb {
 
+// kernel chosen by the last launch_solve on this thread (spline_builder_last_kernel)
+static thread_local char g_last_kernel[96] = "";
+const char *last_kernel() { return g_last_kernel; }
+
 // ------------------------------------------------------------------ host
 namespace {
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+// resolved once, thread-safe (C++11 magic static): concurrent first calls all
+// see the same result instead of racing on a half-written pointer
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
-    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-    static bool tried = false;
-    if (!tried) {
-        tried = true;
+    static const PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
         void *ptr = nullptr;
         cudaDriverEntryPointQueryResult q;
         if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
             q == cudaDriverEntryPointSuccess)
-            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
-    }
+            return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+        return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    }();
     return fn;
+}
+
+// opt-in shared memory per block of each device, queried once (atomic: solves
+// from several host threads may race on the first query)
+int max_smem_of(int dev) {
+    static std::atomic<int> cache[64];
+    int v = (dev >= 0 && dev < 64) ? cache[dev].load(std::memory_order_relaxed) : 0;
+    if (!v) {
+        cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        if (dev >= 0 && dev < 64) cache[dev].store(v, std::memory_order_relaxed);
+    }
+    return v;
 }
 
 int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0) {
@@ -77,6 +94,7 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         kp.bstride = a.bstride;
         kp.pstride = a.pstride;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
+        snprintf(g_last_kernel, sizeof(g_last_kernel), "serial<%s,K=%d>", a.dtype == 0 ? "f64" : "f32", P.K);
         return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
     }
     KParams kp{};
@@ -133,6 +151,7 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         return 5;
     }
     if (!fits) {  // factors + one row do not fit: serial fallback
+        snprintf(g_last_kernel, sizeof(g_last_kernel), "serial<%s,K=%d>", a.dtype == 0 ? "f64" : "f32", P.K);
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
         return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
     }
@@ -140,6 +159,8 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
     const int per_sm = std::max(1, std::min(WARP_MAX_WARPS / wpb, (int)(228 * 1024 / (kp.smem_total + 1024))));
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + wpb - 1) / wpb, (int64_t)num_sms * per_sm));
     // round L up to an instantiated odd length (the plan chose the smallest odd L >= nQ/32)
+    snprintf(g_last_kernel, sizeof(g_last_kernel), "warp<%s,K=%d,L=%d,%s%s>", a.dtype == 0 ? "f64" : "f32", P.K,
+             G.L, kp.bulk ? "BULK" : "DIRECT", kp.adv ? ",ADV" : "");
     if (a.dtype == 0) return launch_warp_f64(P.K, G.L, kp, grid, a.stream, err, errlen);
     return launch_warp_f32(P.K, G.L, kp, grid, a.stream, err, errlen);
 }
@@ -164,12 +185,7 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     const size_t esz = a.dtype == 0 ? 8 : 4;
     int dev = 0;
     cudaGetDevice(&dev);
-    static int max_smem_dev[64] = {0};  // per device, queried once
-    int max_smem = dev >= 0 && dev < 64 ? max_smem_dev[dev] : 0;
-    if (!max_smem) {
-        cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        if (dev >= 0 && dev < 64) max_smem_dev[dev] = max_smem;
-    }
+    const int max_smem = max_smem_of(dev);
 
     // point-contiguous / general strided layouts and the advection step: warp-per-RHS kernel
     if (a.bstride != 1 || a.shift) return launch_warp(P, a, num_sms, max_smem, err, errlen);
@@ -201,6 +217,7 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
         kp.bstride = a.bstride;
         kp.pstride = a.pstride;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
+        snprintf(g_last_kernel, sizeof(g_last_kernel), "serial<%s,K=%d>", a.dtype == 0 ? "f64" : "f32", P.K);
         return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
     }
     const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
@@ -309,6 +326,8 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     }
     const int threads = (kp.ncw + 1) * 32;
     const int grid = (int)std::min<int64_t>((int64_t)kp.ntiles, (int64_t)num_sms);
+    snprintf(g_last_kernel, sizeof(g_last_kernel), "tile<%s,K=%d,R=%d,%s%s>", a.dtype == 0 ? "f64" : "f32", P.K, R,
+             loader == LOAD_TMA ? "TMA" : "DIRECT", cbox ? ",CBOX" : "");
     if (a.dtype == 0) return launch_tile_f64(R, loader, P.K, kp, tm, grid, threads, a.stream, err, errlen);
     return launch_tile_f32(R, loader, P.K, kp, tm, grid, threads, a.stream, err, errlen);
 }
