@@ -41,14 +41,20 @@ def _newer(target: str, deps: list[str]) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False, extra_flags: tuple = (), lib: str = LIB, build_dir: str = BUILD) -> str:
-    """extra_flags / lib / build_dir: diagnostic variants (e.g. -DSB_TRACE) built beside the shipped library."""
+def build(force: bool = False, verbose: bool = False, extra_flags: tuple = (), lib: str = LIB, build_dir: str = BUILD,
+          only: tuple = ()) -> str:
+    """extra_flags / lib / build_dir: diagnostic variants (e.g. -DSB_TRACE) built beside the shipped library.
+    only: compile just these sources in build_dir and link the shipped build's objects for the rest."""
+    default_build = os.path.join(HERE, "_build")
     LIB, BUILD = lib, build_dir
     os.makedirs(BUILD, exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "spline_builder.h")]
     objs, jobs = [], []
     for src, kind in SOURCES:
         path = os.path.join(CSRC, src)
+        if only and src not in only:
+            objs.append(os.path.join(default_build, src.replace("/", "_") + ".o"))
+            continue
         obj = os.path.join(BUILD, src.replace("/", "_") + ".o")
         objs.append(obj)
         if not (force or _newer(obj, [path] + hdrs)):

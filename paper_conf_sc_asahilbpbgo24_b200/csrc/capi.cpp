@@ -76,7 +76,7 @@ int upload(spline_builder *h) {
     for (int d = 0; d < k; ++d) dscale[d] = P.rowscale[P.drow[d]];
     Packer pk;
     // per segment plan: factor arrays in the padded per-segment layout of device.hpp
-    struct SegOff { size_t L[2], U[2], D[2], G[2], H[2], gptr, slot; int LP, nslots; };
+    struct SegOff { size_t F[2], G[2], H[2], gptr, slot; int LP, nslots; };
     SegOff so[3];
     for (int g = 0; g < 3; ++g) {
         const sb::SegPlan &G = P.seg[g];
@@ -113,16 +113,15 @@ int upload(spline_builder *h) {
         }
         const int NS = std::max(1, (int)uniq.size());
         so[g].nslots = NS;
-        std::vector<double> Lr((size_t)K * NS * LP, 0.0), Ur((size_t)K * NS * LP, 0.0), dinv((size_t)NS * LP, 1.0);
+        // one block per slot: [L bands K x LP][U bands K x LP][dinv LP] (device.hpp)
+        const size_t BS = (size_t)(2 * K + 1) * LP;
+        std::vector<double> F(NS * BS, 0.0);
+        for (size_t u = 0; u < (size_t)NS; ++u)
+            for (int i = 0; i < LP; ++i) F[u * BS + (size_t)2 * K * LP + i] = 1.0;  // padding rows: identity
         for (size_t u = 0; u < uniq.size(); ++u) {
             const std::vector<double> &dsd = segdata[uniq[u]];
-            for (int i = 0; i < G.L; ++i) {
-                for (int m = 0; m < K; ++m) {
-                    Lr[((size_t)m * NS + u) * LP + i] = dsd[(size_t)m * G.L + i];
-                    Ur[((size_t)m * NS + u) * LP + i] = dsd[(size_t)(K + m) * G.L + i];
-                }
-                dinv[u * LP + i] = dsd[(size_t)2 * K * G.L + i];
-            }
+            for (int i = 0; i < G.L; ++i)
+                for (int b = 0; b <= 2 * K; ++b) F[u * BS + (size_t)b * LP + i] = dsd[(size_t)b * G.L + i];
         }
         so[g].slot = pk.addv(slot);
         std::vector<int> gptr(S + 1, 0);
@@ -131,9 +130,7 @@ int upload(spline_builder *h) {
             gptr[s] = e;
         }
         if (S > 0) gptr[S] = (int)P.gam_r.size();
-        so[g].L[0] = pk.addv(Lr); so[g].L[1] = pk.addv(conv<float>(Lr));
-        so[g].U[0] = pk.addv(Ur); so[g].U[1] = pk.addv(conv<float>(Ur));
-        so[g].D[0] = pk.addv(dinv); so[g].D[1] = pk.addv(conv<float>(dinv));
+        so[g].F[0] = pk.addv(F); so[g].F[1] = pk.addv(conv<float>(F));
         so[g].G[0] = pk.addv(G.G); so[g].G[1] = pk.addv(conv<float>(G.G));
         so[g].H[0] = pk.addv(G.H); so[g].H[1] = pk.addv(conv<float>(G.H));
         so[g].gptr = pk.addv(gptr);
@@ -153,6 +150,32 @@ int upload(spline_builder *h) {
         auto put = [&](const std::vector<double> &v) { return c == 0 ? pk.addv(v) : pk.addv(conv<float>(v)); };
         oLam[c] = put(P.Lam_v); oGam[c] = put(P.gam_v); oDlu[c] = put(P.dlu); oDs[c] = put(dscale);
     }
+    // tile-kernel corner data (device.hpp): Lambda on a dense column window and
+    // gamma by distinct row
+    int lw_head = 0, lw_tail = 0;
+    for (int c : P.Lam_c) {
+        if (c < nQ / 2) lw_head = std::max(lw_head, c + 1);
+        else lw_tail = std::max(lw_tail, nQ - c);
+    }
+    const int lw_w = lw_head + lw_tail;
+    std::vector<double> lw_v((size_t)std::max(lw_w, 1) * std::max(k, 1), 0.0);
+    for (int d = 0; d < k; ++d)
+        for (int e = P.Lam_ptr[d]; e < P.Lam_ptr[d + 1]; ++e) {
+            const int c = P.Lam_c[e];
+            const int j = c < lw_head ? c : lw_head + (c - (nQ - lw_tail));
+            lw_v[(size_t)j * k + d] = P.Lam_v[e];
+        }
+    std::vector<int> gr_row;
+    std::vector<double> gr_v;
+    for (size_t e = 0; e < P.gam_r.size(); ++e) {
+        if (gr_row.empty() || gr_row.back() != P.gam_r[e]) {
+            gr_row.push_back(P.gam_r[e]);
+            gr_v.resize(gr_v.size() + k, 0.0);
+        }
+        gr_v[(gr_row.size() - 1) * k + P.gam_c[e]] += P.gam_v[e];
+    }
+    size_t o_lw[2] = {pk.addv(lw_v), pk.addv(conv<float>(lw_v))};
+    size_t o_grr = pk.addv(gr_row), o_grv[2] = {pk.addv(gr_v), pk.addv(conv<float>(gr_v))};
     size_t o_lamptr = pk.addv(P.Lam_ptr), o_lamc = pk.addv(P.Lam_c), o_gamr = pk.addv(P.gam_r),
            o_gamc = pk.addv(P.gam_c), o_dpiv = pk.addv(P.dpiv), o_drow = pk.addv(P.drow);
     h->blob_bytes = std::max<size_t>(pk.bytes.size(), 16);
@@ -178,6 +201,11 @@ int upload(spline_builder *h) {
         for (int r : P.drow) note(r);
         for (int c : P.Lam_c) note(P.s_lo + c);
         d.corner_rows = k > 0 ? std::max(head, tail) : 0;
+        d.gam_head = d.gam_tail = 0;
+        for (int r : P.gam_r) {
+            if (r < nQ / 2) d.gam_head = std::max(d.gam_head, r + 1);
+            else d.gam_tail = std::max(d.gam_tail, nQ - r);
+        }
     }
     for (int c = 0; c < 2; ++c) {
         d.lam_v[c] = at(oLam[c]); d.gam_v[c] = at(oGam[c]); d.dlu[c] = at(oDlu[c]); d.dscale[c] = at(oDs[c]);
@@ -189,7 +217,7 @@ int upload(spline_builder *h) {
         ds.L = G.L; ds.S = G.S; ds.LP = so[g].LP; ds.carry_f = G.carry_f; ds.carry_b = G.carry_b;
         ds.nslots = so[g].nslots; ds.slot = (const int *)at(so[g].slot);
         for (int c = 0; c < 2; ++c) {
-            ds.Lr[c] = at(so[g].L[c]); ds.Ur[c] = at(so[g].U[c]); ds.dinv[c] = at(so[g].D[c]);
+            ds.F[c] = at(so[g].F[c]);
             ds.G[c] = at(so[g].G[c]); ds.H[c] = at(so[g].H[c]);
         }
         ds.gptr = (const int *)at(so[g].gptr);
@@ -200,6 +228,9 @@ int upload(spline_builder *h) {
     d.adv_tbl = (const int *)at(oTbl); d.adv_nbkt = (int)P.adv_tbl.size(); d.adv_steps = P.adv_steps;
     d.adv_bscale = P.xe.empty() ? 0.0 : (double)P.adv_tbl.size() / (P.xb[P.N] - P.xb[0]);
     d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
+    d.lw_head = lw_head; d.lw_tail = lw_tail; d.gr_n = (int)gr_row.size();
+    d.gr_row = (const int *)at(o_grr);
+    for (int c = 0; c < 2; ++c) { d.lw_v[c] = at(o_lw[c]); d.gr_v[c] = at(o_grv[c]); }
     d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);
     d.dpiv = (const int *)at(o_dpiv); d.drow = (const int *)at(o_drow);
     return 0;

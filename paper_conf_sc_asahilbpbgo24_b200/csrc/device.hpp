@@ -7,18 +7,20 @@
 namespace sb {
 
 // Segment plan of one kernel family: Q padded to S*L rows, split into S
-// register segments of L rows.  Factor arrays are stored per segment with a
-// padded pitch LP (bank-conflict-free broadcast reads, 16-B aligned pairs):
-//   L(a+i, a+i-1-m)  at Lr[(m*NS + slot[s])*LP + i]      (a = s*L, NS = nslots)
-//   U'(a+i, a+i+1+m) at Ur[(m*NS + slot[s])*LP + i]
-//   dinv(a+i)        at dinv[slot[s]*LP + i]               (1 on padding rows)
+// register segments of L rows.  The factors of a segment form one block of
+// (2K+1) rows of pitch LP (16-B aligned pairs; tile kernels LP = L+2 fp64 /
+// L+4 fp32, warp kernel LP = L odd), so a thread needs ONE base address and
+// every factor offset is a compile-time immediate:
+//   F + slot[s]*(2K+1)*LP:  L(a+i, a+i-1-m)  at [m*LP + i]        (a = s*L)
+//                           U'(a+i, a+i+1+m) at [(K+m)*LP + i]
+//                           dinv(a+i)        at [2K*LP + i]         (1 on padding rows)
 // Segments with bitwise-identical factors share a slot (broadcast reads).
 // Floating-point arrays exist in fp64 ([0]) and fp32 ([1]).
 struct DevSeg {
     int L, S, LP, carry_f, carry_b;
     int nslots;               // distinct factor blocks; segment s reads block slot[s]
     const int *slot;
-    const void *Lr[2], *Ur[2], *dinv[2];
+    const void *F[2];         // nslots factor blocks of (2K+1)*LP, fp64 [0] / fp32 [1]
     const void *G[2], *H[2];  // S*K*K forward / backward segment transfer matrices
     const int *gptr;          // S+1: gamma COO entries of segment s are [gptr[s], gptr[s+1])
 };
@@ -29,6 +31,7 @@ struct DevPlan {
     int n, nQ, s_lo, k, K;   // order, Q order, Q offset, delta order, kernel band
     int lam_nnz, gam_nnz;    // Lambda CSR / gamma COO sizes
     int corner_rows;         // rows [0,c) and [n-c,n) hold every row the corner reads (0: none/unbounded)
+    int gam_head, gam_tail;  // gamma rows lie in Q rows [0, gam_head) and [nQ-gam_tail, nQ)
     const void *lam_v[2], *gam_v[2], *dlu[2], *dscale[2];
     const void *rowf[2];     // nQ x (2K+1): L(i,i-1..i-K), U'(i,i+1..i+K), dinv(i) -- serial fallback
     int p, N, periodic;      // spline degree, cells, periodic flag (advection / evaluation)
@@ -40,6 +43,14 @@ struct DevPlan {
     int adv_nbkt, adv_steps;
     double adv_bscale;       // adv_nbkt / (x_N - x_0)
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
+    // Tile-kernel corner (dense, so every shared-memory load is independent of
+    // the others -- no column-index load in front of each b load):
+    //   Lambda on a column window: Q columns [0, lw_head) then [nQ-lw_tail, nQ),
+    //   lw_v[j*k + d] = Lambda(d, column j of the window) (0 where dropped);
+    //   gamma by distinct row: Q row gr_row[g], gr_v[g*k + d] = gamma(row, d).
+    int lw_head, lw_tail, gr_n;
+    const void *lw_v[2], *gr_v[2];
+    const int *gr_row;
     DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),
                              // [2] warp-per-RHS kernel (odd L; S == 0 if unavailable)
 };

@@ -462,8 +462,10 @@ void plan_solve_cpu(const Plan &P, double *rhs, int64_t batch, int64_t bstride, 
     }
 }
 
-Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi) {
+Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi,
+                  int flags) {
     P = Plan();
+    P.dev_update = (flags & PLAN_DEVICE_UPDATE) != 0;
     if (degree < 1 || degree > 5) return {1, "degree must be in 1..5"};
     // bc < 16: both ends alike; else lo | (hi << 4) (mixed, R13)
     int bc_lo = bc, bc_hi = bc;
@@ -505,42 +507,42 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         if (!(P.h[c] > 0.0) || !std::isfinite(P.h[c])) return {1, "breakpoints must be strictly increasing"};
     }
     Space S{p, bc == PERIODIC ? PERIODIC : GREVILLE, N, n, P.nbc, P.h.data()};  // clamped knots unless periodic
-    // rows
-    std::vector<RowPt> rows(n);
-    P.rowscale.assign(n, 1.0);
+    // rows: mesh-independent descriptors first (device refactorisation reuses them)
+    P.rowdesc.clear();
     if (mixed) {
         // derivative rows at a Hermite end; the Greville abscissae minus the nbc
         // next to a Hermite end (the end point itself stays)
-        int r = 0;
-        for (int d = 1; d <= P.nbc_lo; ++d) { rows[r] = RowPt{S.span_of_cell(0), 0.0, d}; P.rowscale[r] = std::pow(P.h[0], d); ++r; }
+        for (int d = 1; d <= P.nbc_lo; ++d) P.rowdesc.push_back({ROW_DER0, 0, d});
         for (int j = 0; j < n; ++j) {
             if (j >= 1 && j <= P.nbc_lo) continue;
             if (j >= n - 1 - P.nbc_hi && j <= n - 2) continue;
-            rows[r++] = greville(S, j);
+            P.rowdesc.push_back({ROW_GREVILLE, j, 0});
         }
-        for (int d = 1; d <= P.nbc_hi; ++d) {
-            rows[r] = RowPt{S.span_of_cell(N - 1), P.h[N - 1], d};
-            P.rowscale[r] = std::pow(P.h[N - 1], d);
-            ++r;
-        }
-        if (r != n) return {1, "mixed boundary rows do not add up"};
+        for (int d = 1; d <= P.nbc_hi; ++d) P.rowdesc.push_back({ROW_DERN, 0, d});
+        if ((int)P.rowdesc.size() != n) return {1, "mixed boundary rows do not add up"};
     } else if (bc != HERMITE) {
-        for (int j = 0; j < n; ++j) rows[j] = greville(S, j);
+        for (int j = 0; j < n; ++j) P.rowdesc.push_back({ROW_GREVILLE, j, 0});
     } else {
-        int r = 0;
-        for (int d = 1; d <= P.nbc; ++d) { rows[r] = RowPt{S.span_of_cell(0), 0.0, d}; P.rowscale[r] = std::pow(P.h[0], d); ++r; }
+        for (int d = 1; d <= P.nbc; ++d) P.rowdesc.push_back({ROW_DER0, 0, d});
         if (p % 2) {
-            for (int i = 0; i <= N; ++i) {
-                rows[r] = i < N ? RowPt{S.span_of_cell(i), 0.0, 0} : RowPt{S.span_of_cell(N - 1), P.h[N - 1], 0};
-                ++r;
-            }
+            for (int i = 0; i < N; ++i) P.rowdesc.push_back({ROW_BREAK, i, 0});
+            P.rowdesc.push_back({ROW_END, N, 0});
         } else {
-            for (int c = 0; c < N; ++c) { rows[r] = RowPt{S.span_of_cell(c), 0.5 * P.h[c], 0}; ++r; }
+            for (int c = 0; c < N; ++c) P.rowdesc.push_back({ROW_MID, c, 0});
         }
-        for (int d = 1; d <= P.nbc; ++d) {
-            rows[r] = RowPt{S.span_of_cell(N - 1), P.h[N - 1], d};
-            P.rowscale[r] = std::pow(P.h[N - 1], d);
-            ++r;
+        for (int d = 1; d <= P.nbc; ++d) P.rowdesc.push_back({ROW_DERN, 0, d});
+    }
+    std::vector<RowPt> rows(n);
+    P.rowscale.assign(n, 1.0);
+    for (int i = 0; i < n; ++i) {
+        const RowDesc &d = P.rowdesc[i];
+        switch (d.kind) {
+            case ROW_GREVILLE: rows[i] = greville(S, d.idx); break;
+            case ROW_BREAK: rows[i] = RowPt{S.span_of_cell(d.idx), 0.0, 0}; break;
+            case ROW_END: rows[i] = RowPt{S.span_of_cell(N - 1), P.h[N - 1], 0}; break;
+            case ROW_MID: rows[i] = RowPt{S.span_of_cell(d.idx), 0.5 * P.h[d.idx], 0}; break;
+            case ROW_DER0: rows[i] = RowPt{S.span_of_cell(0), 0.0, d.deriv}; P.rowscale[i] = std::pow(P.h[0], d.deriv); break;
+            default: rows[i] = RowPt{S.span_of_cell(N - 1), P.h[N - 1], d.deriv}; P.rowscale[i] = std::pow(P.h[N - 1], d.deriv); break;
         }
     }
     // breakpoints and row positions (advection / evaluation data)

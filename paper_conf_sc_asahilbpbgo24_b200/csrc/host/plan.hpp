@@ -21,6 +21,24 @@ constexpr int KMAX_BAND = 4;          // largest Q half-band the kernels are bui
 constexpr int KMAX_DELTA = 32;        // largest delta' order
 constexpr double CORNER_DROP = 1e-14; // keep |beta|, |Lambda| > 1e-14 (DESIGN R4)
 
+// What an interpolation row is, independent of the mesh (device-side
+// refactorisation recomputes its point for new breakpoints):
+//   GREVILLE  Greville abscissa of basis idx        BREAK  value at x_idx (idx < N)
+//   END       value at x_N                           MID    value at the midpoint of cell idx
+//   DER0/DERN derivative of order deriv at x_0 / x_N
+enum RowKind { ROW_GREVILLE = 0, ROW_BREAK = 1, ROW_END = 2, ROW_MID = 3, ROW_DER0 = 4, ROW_DERN = 5 };
+struct RowDesc {
+    int kind, idx, deriv;
+};
+
+// build_plan flags
+enum PlanFlags {
+    PLAN_DEVICE_UPDATE = 1  // structure frozen for device-side refactorisation: corner patterns dilated by
+                            // CORNER_MARGIN, carry walks one segment deeper, no slot sharing, generic
+                            // (non-uniform) advection geometry with a 2x finer bucket table
+};
+constexpr int CORNER_MARGIN = 16;  // Lambda columns / gamma rows kept around the create-time pattern
+
 struct SparseRow {
     std::vector<int> col;
     std::vector<double> val;
@@ -49,6 +67,8 @@ struct Plan {
     int adv_steps = 0;              // forward steps from the bucket's cell to the point's cell (<= 2 typically)
     std::vector<int> adv_tbl;       // periodic: buckets of [x_0, x_N) no wider than the smallest cell -> cell
     std::vector<double> adv_rcp;    // periodic: 1/(t_{m+w} - t_m) at [(m+p)*(p|1) + w-1], m in [-p, N+p), w = 1..p
+    std::vector<RowDesc> rowdesc;   // n row descriptors (mesh independent)
+    bool dev_update = false;        // PLAN_DEVICE_UPDATE
     std::vector<SparseRow> A;       // equilibrated collocation matrix rows
     std::vector<double> rowscale;   // A_eq = diag(rowscale) * A_raw
     // ---- Schur split (Eq. 3)
@@ -83,7 +103,8 @@ struct Status {
 
 // Build the spline space, the (equilibrated) collocation matrix, choose the
 // split, factor, compute corners and segment data.  split_lo/hi = -1: default.
-Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi);
+Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots, int split_lo, int split_hi,
+                  int flags = 0);
 
 // Algorithm 1 on the CPU with the plan's factors (serial, fp64), in the same
 // order as the kernels (Lambda / gamma form).  Used by create's self-check.

@@ -77,6 +77,8 @@ struct KParams {
     int corner_arrive_mask;          // boxes without a compute-warp reader: the corner warp frees them
     int cbox;                        // rows of each corner box (0: corner reads the main tile)
     // dynamic shared memory offsets (bytes)
+    int off_lw, off_grr, off_grv;    // tile corner: Lambda window, gamma rows (DevPlan::lw_*, gr_*)
+    int gbox_mask;                   // tile kernel: TMA boxes holding gamma rows (the corner warp patches them)
     int off_buf, off_L, off_U, off_dinv, off_G, off_H, off_fend, off_bbeg, off_x1, off_lamptr, off_lamc, off_lamv,
         off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, off_cbuf,
         smem_total;
@@ -276,9 +278,11 @@ __device__ __forceinline__ void bwd_local(C (&v)[L][NV], const C *fU, const C *f
 
 // backward correction chain c_i = -sum_m U'(i,i+1+m) c_{i+1+m}, c(a+L+m) = co[m];  x_i += c_i.
 // STORE: row i is final once corrected, so it goes to HBM right there (one
-// NV-wide vector at dst + i*ps, rows i < nvalid): the stores trickle out under the chain's
-// FMA latency instead of leaving every warp of the tile in one burst.
-template <typename C, int K, int L, int NV, bool PAIRS, bool STORE = false, typename T = C>
+// NV-wide vector per row): the stores trickle out under the chain's FMA latency
+// instead of leaving every warp of the tile in one burst.  dst points at row
+// L-1 of this segment and walks back by ps per row (one 64-bit add per row,
+// not a multiply); rows i >= nvalid are not stored (PRED only: the last segment).
+template <typename C, int K, int L, int NV, bool PAIRS, bool STORE = false, bool PRED = false, typename T = C>
 __device__ __forceinline__ void bwd_correct(C (&v)[L][NV], const C *fU, int ms, C (&co)[K][NV],
                                             T *dst = nullptr, int64_t ps = 0, int nvalid = 0) {
     using V = typename std::conditional<NV == 1, T,
@@ -301,12 +305,15 @@ __device__ __forceinline__ void bwd_correct(C (&v)[L][NV], const C *fU, int ms, 
                 co[0][q] = c;
                 v[i + h][q] += c;
             }
-            if (STORE && i + h < nvalid) {
-                V w;
-                T *pw = reinterpret_cast<T *>(&w);
+            if constexpr (STORE) {
+                if (!PRED || i + h < nvalid) {
+                    V w;
+                    T *pw = reinterpret_cast<T *>(&w);
 #pragma unroll
-                for (int q = 0; q < NV; ++q) pw[q] = (T)v[i + h][q];
-                __stcs(reinterpret_cast<V *>(dst + (int64_t)(i + h) * ps), w);
+                    for (int q = 0; q < NV; ++q) pw[q] = (T)v[i + h][q];
+                    __stcs(reinterpret_cast<V *>(dst), w);
+                }
+                dst -= ps;
             }
         }
     }
@@ -373,28 +380,26 @@ __device__ __forceinline__ void wgetrs_reg(C (&x)[KR], const C *lu, const int *p
 // load/store loop: the copies stream at L2 bandwidth and cost the CTA a
 // single wait.  Every array starts 16-B aligned in the blob and in shared
 // memory and its size is rounded up to 16 B (the blob pads each array).
-struct StageList {
-    static constexpr int MAXN = 24;
-    void *dst[MAXN];
-    const void *src[MAXN];
-    uint32_t bytes[MAXN];
-    int n = 0;
-    uint32_t total = 0;
-    __device__ __forceinline__ void add(void *d, const void *sr, size_t nb) {
-        const uint32_t b16 = (uint32_t)((nb + 15) & ~(size_t)15);
-        if (b16 == 0) return;
-        dst[n] = d; src[n] = sr; bytes[n] = b16; ++n;
-        total += b16;
-    }
-};
+// Each copy raises the barrier's expected transaction count itself
+// (mbarrier.expect_tx), and one arrive closes the list, so no list of copies
+// is kept (a local array of them would live on the stack).
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *mbar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                      smem_u32(dst)),
                  "l"(src), "r"(bytes), "r"(smem_u32(mbar))
                  : "memory");
 }
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *m, uint32_t bytes) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(m)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void stage_one(void *dst, const void *src, size_t nb, uint64_t *bar) {
+    const uint32_t b16 = (uint32_t)((nb + 15) & ~(size_t)15);
+    if (b16 == 0) return;
+    mbar_expect_tx(bar, b16);
+    bulk_g2s(dst, src, b16, bar);
+}
 
-// one thread: arm the barrier with the total and issue every copy
+// one thread: issue every copy, then the single arrival that lets the phase complete
 template <typename C, int K>
 __device__ __forceinline__ void stage_constants_issue(const KParams &p, const DevSeg &G, unsigned char *smem,
                                                       uint64_t *cbar) {
@@ -402,34 +407,166 @@ __device__ __forceinline__ void stage_constants_issue(const KParams &p, const De
     const DevPlan &P = p.P;
     const int k = P.k, S = G.S;
     const size_t esz = sizeof(C);
-    const size_t nrec = (size_t)K * G.nslots * G.LP;
-    StageList L;
-    L.add(smem + p.off_L, G.Lr[CI], nrec * esz);
-    L.add(smem + p.off_U, G.Ur[CI], nrec * esz);
-    L.add(smem + p.off_dinv, G.dinv[CI], (size_t)G.nslots * G.LP * esz);
-    L.add(smem + p.off_G, G.G[CI], (size_t)S * K * K * esz);
-    L.add(smem + p.off_H, G.H[CI], (size_t)S * K * K * esz);
-    L.add(smem + p.off_lamptr, P.lam_ptr, (size_t)(k + 1) * 4);
-    L.add(smem + p.off_lamc, P.lam_c, (size_t)P.lam_nnz * 4);
-    L.add(smem + p.off_lamv, P.lam_v[CI], (size_t)P.lam_nnz * esz);
-    L.add(smem + p.off_gamr, P.gam_r, (size_t)P.gam_nnz * 4);
-    L.add(smem + p.off_gamc, P.gam_c, (size_t)P.gam_nnz * 4);
-    L.add(smem + p.off_gamv, P.gam_v[CI], (size_t)P.gam_nnz * esz);
-    L.add(smem + p.off_gptr, G.gptr, (size_t)(S + 1) * 4);
-    L.add(smem + p.off_dlu, P.dlu[CI], (size_t)k * k * esz);
-    L.add(smem + p.off_dpiv, P.dpiv, (size_t)k * 4);
-    L.add(smem + p.off_dscale, P.dscale[CI], (size_t)k * esz);
-    L.add(smem + p.off_drow, P.drow, (size_t)k * 4);
+    stage_one(smem + p.off_L, G.F[CI], (size_t)G.nslots * (2 * K + 1) * G.LP * esz, cbar);
+    stage_one(smem + p.off_G, G.G[CI], (size_t)S * K * K * esz, cbar);
+    stage_one(smem + p.off_H, G.H[CI], (size_t)S * K * K * esz, cbar);
+    stage_one(smem + p.off_lamptr, P.lam_ptr, (size_t)(k + 1) * 4, cbar);
+    stage_one(smem + p.off_lamc, P.lam_c, (size_t)P.lam_nnz * 4, cbar);
+    stage_one(smem + p.off_lamv, P.lam_v[CI], (size_t)P.lam_nnz * esz, cbar);
+    stage_one(smem + p.off_lw, P.lw_v[CI], (size_t)(P.lw_head + P.lw_tail) * k * esz, cbar);
+    stage_one(smem + p.off_grr, P.gr_row, (size_t)P.gr_n * 4, cbar);
+    stage_one(smem + p.off_grv, P.gr_v[CI], (size_t)P.gr_n * k * esz, cbar);
+    stage_one(smem + p.off_gamr, P.gam_r, (size_t)P.gam_nnz * 4, cbar);
+    stage_one(smem + p.off_gamc, P.gam_c, (size_t)P.gam_nnz * 4, cbar);
+    stage_one(smem + p.off_gamv, P.gam_v[CI], (size_t)P.gam_nnz * esz, cbar);
+    stage_one(smem + p.off_gptr, G.gptr, (size_t)(S + 1) * 4, cbar);
+    stage_one(smem + p.off_dlu, P.dlu[CI], (size_t)k * k * esz, cbar);
+    stage_one(smem + p.off_dpiv, P.dpiv, (size_t)k * 4, cbar);
+    stage_one(smem + p.off_dscale, P.dscale[CI], (size_t)k * esz, cbar);
+    stage_one(smem + p.off_drow, P.drow, (size_t)k * 4, cbar);
     if (p.adv && !P.adv_uniform) {  // advection geometry: xe | xi | rcp | bucket table, each 16-B aligned
         const GeoLayout gl(P);
         double *sgeo = reinterpret_cast<double *>(smem + p.off_geo);
-        L.add(sgeo, P.xe, (size_t)(P.N + 2 * P.p + 1) * 8);
-        L.add(sgeo + gl.o_xi, P.xi, (size_t)P.n * 8);
-        L.add(sgeo + gl.o_rc, P.adv_rcp, (size_t)(P.N + 2 * P.p) * (P.p | 1) * 8);
-        L.add(sgeo + gl.o_tbl, P.adv_tbl, (size_t)P.adv_nbkt * 4);
+        stage_one(sgeo, P.xe, (size_t)(P.N + 2 * P.p + 1) * 8, cbar);
+        stage_one(sgeo + gl.o_xi, P.xi, (size_t)P.n * 8, cbar);
+        stage_one(sgeo + gl.o_rc, P.adv_rcp, (size_t)(P.N + 2 * P.p) * (P.p | 1) * 8, cbar);
+        stage_one(sgeo + gl.o_tbl, P.adv_tbl, (size_t)P.adv_nbkt * 4, cbar);
     }
-    mbar_arrive_expect_tx(cbar, L.total);
-    for (int i = 0; i < L.n; ++i) bulk_g2s(L.dst[i], L.src[i], L.bytes[i], cbar);
+    mbar_arrive(cbar);
+}
+
+// bulk (non-tensor) copies and the generic->async proxy fence
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *mbar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(mbar))
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_store(void *dst, const void *src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ---------------------------------------------------- tile-kernel corner
+// x1 = delta'^{-1} (s1 b1 - Lambda b0) for one tile (one RHS per lane pair),
+// run by the corner/producer warp one tile ahead of the compute warps.
+template <typename C, typename T> struct CornerCtx {
+    int part, rr, s_lo, it, nbox, gbox_mask, lh, lw, tail0, gr_n;
+    const C *slw, *sgrv, *sdlu, *sdscale;
+    const int *sgrr, *sdrow, *sdpiv;
+    uint64_t *full, *gready;
+    T *buf;
+    C *sx1;       // this lane's x1 slot (DIRECT loader / k > 8)
+    T *gout;      // column of this RHS in HBM (nullptr: RHS beyond the batch)
+    int64_t ps;
+    bool patch;   // gamma patched into the shared-memory tile by this warp (else x1 -> sx1)
+};
+
+// TMA path: the corner warp applies b0 -= gamma x1 to the gamma rows of the
+// tile in the shared-memory boxes once they have landed, so the compute warps
+// neither wait for x1 nor select rows by a runtime index.  All loads first,
+// then all stores; then the generic->async proxy fence (the boxes are refilled
+// by TMA later) and the arrival on gready.
+template <typename C, typename T, int R>
+__device__ __forceinline__ void patch_gamma_done(const CornerCtx<C, T> &cx) {
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (cx.part == 0) mbar_arrive(cx.gready + (cx.it & 1));
+}
+template <typename C, typename T, int R>
+__device__ __forceinline__ void patch_gamma_wait(const CornerCtx<C, T> &cx) {
+    for (int c = 0; c < cx.nbox; ++c)
+        if ((cx.gbox_mask >> c) & 1) mbar_wait(cx.full + c, cx.it & 1);
+}
+template <typename C, typename T, int R, int KC>
+__device__ __forceinline__ void patch_gamma_reg(const CornerCtx<C, T> &cx, const C (&xr)[KC]) {
+    patch_gamma_wait<C, T, R>(cx);
+    if (cx.part == 0) {
+        constexpr int GB = 8;
+        for (int g0 = 0; g0 < cx.gr_n; g0 += GB) {
+            int off[GB];
+            C val[GB];
+#pragma unroll
+            for (int g = 0; g < GB; ++g) {
+                off[g] = g0 + g < cx.gr_n ? (cx.s_lo + cx.sgrr[g0 + g]) * R + cx.rr : -1;
+                val[g] = off[g] >= 0 ? (C)cx.buf[off[g]] : C(0);
+            }
+#pragma unroll
+            for (int g = 0; g < GB; ++g) {
+                C acc = val[g];
+#pragma unroll
+                for (int d = 0; d < KC; ++d) acc = fma(-cx.sgrv[(g0 + g) * KC + d], xr[d], acc);
+                if (off[g] >= 0) cx.buf[off[g]] = (T)acc;
+            }
+        }
+    }
+    patch_gamma_done<C, T, R>(cx);
+}
+template <typename C, typename T, int R>
+__device__ __forceinline__ void patch_gamma_smem(const CornerCtx<C, T> &cx, int k) {
+    patch_gamma_wait<C, T, R>(cx);
+    if (cx.part == 0)
+        for (int g = 0; g < cx.gr_n; ++g) {
+            T *q = cx.buf + (cx.s_lo + cx.sgrr[g]) * R + cx.rr;
+            C acc = (C)*q;
+            for (int d = 0; d < k; ++d) acc = fma(-cx.sgrv[g * k + d], cx.sx1[d], acc);
+            *q = (T)acc;
+        }
+    patch_gamma_done<C, T, R>(cx);
+}
+
+// k = KC <= 8: Lambda on its dense column window (each b row loaded once for
+// all KC rows; loads in independent batches), xor-shuffle over the CPR lanes
+// of a RHS, getrs on registers, delta rows of x to HBM, gamma patch (TMA) or
+// x1 to shared memory (DIRECT loader: the compute warps apply gamma).
+template <typename C, typename T, int KC, int R, typename LDB>
+__device__ __forceinline__ void tile_corner(const CornerCtx<C, T> &cx, LDB ldb) {
+    constexpr int CPR = 32 / R;
+    C xr[KC];
+#pragma unroll
+    for (int d = 0; d < KC; ++d) xr[d] = C(0);
+    constexpr int JB = 8;
+    for (int j0 = cx.part; j0 < cx.lw; j0 += JB * CPR) {
+        C b[JB];
+#pragma unroll
+        for (int u = 0; u < JB; ++u) {
+            const int j = j0 + u * CPR;
+            b[u] = j < cx.lw ? ldb(j < cx.lh ? cx.s_lo + j : cx.tail0 + j) : C(0);
+        }
+#pragma unroll
+        for (int u = 0; u < JB; ++u) {
+            const int j = j0 + u * CPR;
+            if (j < cx.lw) {
+                const C *lv = cx.slw + j * KC;
+#pragma unroll
+                for (int d = 0; d < KC; ++d) xr[d] = fma(-lv[d], b[u], xr[d]);
+            }
+        }
+    }
+#pragma unroll
+    for (int d = 0; d < KC; ++d) {
+        C acc = xr[d];
+#pragma unroll
+        for (int off = R; off < 32; off *= 2) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        xr[d] = fma(ldb(cx.sdrow[d]), cx.sdscale[d], acc);
+    }
+    wgetrs_reg<C, KC>(xr, cx.sdlu, cx.sdpiv, KC);
+    if (cx.part == 0 && cx.gout)
+#pragma unroll
+        for (int d = 0; d < KC; ++d) __stcs(cx.gout + (int64_t)cx.sdrow[d] * cx.ps, (T)xr[d]);
+    if (cx.patch) {
+        patch_gamma_reg<C, T, R, KC>(cx, xr);
+    } else if (cx.part == 0) {
+#pragma unroll
+        for (int d = 0; d < KC; ++d) cx.sx1[d] = xr[d];
+    }
 }
 
 // ========================================================= tile kernel
@@ -457,14 +594,20 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const DevPlan &P = p.P;
     const DevSeg &G = P.seg[CI];
 
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int S = G.S, LP = G.LP, nQ = P.nQ, k = P.k, s_lo = P.s_lo;
+    const int S = G.S, nQ = P.nQ, k = P.k, s_lo = P.s_lo;
     const int ncw = p.ncw, nbox = p.nbox, boxr = p.boxr;
-    const int ms = G.nslots * LP;  // band stride of the factor arrays
+    // The corner/producer warp runs on hardware warp 0: the warp schedulers favour
+    // older warps, and the corner's short dependent chains (x1 for the next tile)
+    // must not be starved by the compute warps (as the youngest warp it finished
+    // x1 only just before the gamma warps needed it).  Logical numbering: compute
+    // warps 0..ncw-1 (hardware warps 1..ncw), corner warp ncw.
+    const int hwarp = (int)(threadIdx.x >> 5), lane = (int)(threadIdx.x & 31);
+    const int warp = hwarp == 0 ? ncw : hwarp - 1;
+    const int tid = warp * 32 + lane;
+    constexpr int LP = L + (sizeof(T) == 8 ? 2 : 4);  // factor pitch (capi.cpp upload; checked at launch)
+    constexpr int ms = LP;                            // band stride inside a segment's factor block
 
-    C *sL = reinterpret_cast<C *>(smem + p.off_L);
-    C *sU = reinterpret_cast<C *>(smem + p.off_U);
-    C *sdinv = reinterpret_cast<C *>(smem + p.off_dinv);
+    C *sF = reinterpret_cast<C *>(smem + p.off_L);  // factor blocks (device.hpp DevSeg)
     C *sG = reinterpret_cast<C *>(smem + p.off_G);
     C *sH = reinterpret_cast<C *>(smem + p.off_H);
     C *sfend = reinterpret_cast<C *>(smem + p.off_fend);
@@ -473,6 +616,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const int *slamptr = reinterpret_cast<const int *>(smem + p.off_lamptr);
     const int *slamc = reinterpret_cast<const int *>(smem + p.off_lamc);
     const C *slamv = reinterpret_cast<const C *>(smem + p.off_lamv);
+    const C *slw = reinterpret_cast<const C *>(smem + p.off_lw);
+    const int *sgrr = reinterpret_cast<const int *>(smem + p.off_grr);
+    const C *sgrv = reinterpret_cast<const C *>(smem + p.off_grv);
     const int *sgamr = reinterpret_cast<const int *>(smem + p.off_gamr);
     const int *sgamc = reinterpret_cast<const int *>(smem + p.off_gamc);
     const C *sgamv = reinterpret_cast<const C *>(smem + p.off_gamv);
@@ -484,11 +630,16 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + p.off_mbar);
     uint64_t *empty = full + NBOXMAX;
     uint64_t *x1full = empty + NBOXMAX;
-    uint64_t *cfull = x1full + 2;  // corner boxes, double-buffered
+    uint64_t *cfull = x1full + 2;  // corner boxes, double-buffered (+ [2]: constants staged)
+    uint64_t *gready = cfull + 3;  // TMA path: gamma rows of the tile patched in smem, double-buffered
     T *buf = reinterpret_cast<T *>(smem + p.off_buf);
     T *cbuf = reinterpret_cast<T *>(smem + p.off_cbuf);  // [2][2 boxes][cbox rows][R]
     const int cbox = p.cbox;
     const bool use_cbox = LOADER == LOAD_TMA && cbox > 0;
+    // gamma patched in shared memory by the corner warp: only when x1 is computed a
+    // tile ahead from the corner boxes (without them the gamma warps would wait for
+    // x1 before they even load their rows)
+    const bool gpatch = use_cbox;
     T *gout = reinterpret_cast<T *>(p.rhs);
     const int64_t ps = p.pstride;
     const uint32_t box_bytes = (uint32_t)(boxr * R * sizeof(T));
@@ -503,6 +654,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         mbar_init(cfull + 0, 1);
         mbar_init(cfull + 1, 1);
         mbar_init(cfull + 2, 1);  // constants staged
+        mbar_init(gready + 0, R);  // every patching corner lane arrives
+        mbar_init(gready + 1, R);
         fence_mbar_init();
         if (LOADER == LOAD_TMA) prefetch_tmap(&tmap);
         if (use_cbox) prefetch_tmap(&tmap_c);
@@ -540,6 +693,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                     }
                     if (use_cbox && tile + (int)gridDim.x < p.ntiles) issue_cbox(tile + gridDim.x, (it + 1) & 1);
                 }
+                // every lane passes lane 0's empty waits: the compute warps have loaded
+                // tile it-1, so they are done with tile it-2 and its x1 buffer (it & 1)
+                __syncwarp();
                 SB_TR(8);
                 if (use_cbox) mbar_wait(cfull + (it & 1), (it >> 1) & 1);
                 else
@@ -559,30 +715,46 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 }
                 return clive ? (C)ccolp[(int64_t)row * ps] : C(0);
             };
-            C *x1 = sx1 + (it & 1) * R * k + rr * k;
-            for (int d = 0; d < k; ++d) {
-                C acc = part == 0 ? ldb(sdrow[d]) * sdscale[d] : C(0);
-                int e = slamptr[d] + part;
-                const int e1 = slamptr[d + 1];
-                // 4 independent partial sums keep the dependent smem loads in flight
-                C a1 = C(0), a2 = C(0), a3 = C(0);
-                for (; e + 3 * CPR < e1; e += 4 * CPR) {
-                    acc = fma(-slamv[e], ldb(s_lo + slamc[e]), acc);
-                    a1 = fma(-slamv[e + CPR], ldb(s_lo + slamc[e + CPR]), a1);
-                    a2 = fma(-slamv[e + 2 * CPR], ldb(s_lo + slamc[e + 2 * CPR]), a2);
-                    a3 = fma(-slamv[e + 3 * CPR], ldb(s_lo + slamc[e + 3 * CPR]), a3);
+            CornerCtx<C, T> cx;
+            cx.part = part; cx.rr = rr; cx.s_lo = s_lo; cx.it = it; cx.nbox = nbox; cx.gbox_mask = p.gbox_mask;
+            cx.lh = P.lw_head; cx.lw = P.lw_head + P.lw_tail; cx.tail0 = s_lo + nQ - P.lw_tail - P.lw_head;
+            cx.gr_n = P.gr_n; cx.slw = slw; cx.sgrv = sgrv; cx.sdlu = sdlu; cx.sdscale = sdscale;
+            cx.sgrr = sgrr; cx.sdrow = sdrow; cx.sdpiv = sdpiv; cx.full = full; cx.gready = gready; cx.buf = buf;
+            cx.sx1 = sx1 + (it & 1) * R * k + rr * k;
+            cx.gout = clive ? gs + ccol * p.bstride : nullptr; cx.ps = ps;
+            cx.patch = gpatch;
+            if (k >= 1 && k <= WCORNER_KREG) {
+                // x1 in registers with k a compile-time constant (every instruction of the
+                // corner warp costs ~4 issue cycles next to the compute warps)
+                switch (k) {
+                    case 1: tile_corner<C, T, 1, R>(cx, ldb); break;
+                    case 2: tile_corner<C, T, 2, R>(cx, ldb); break;
+                    case 3: tile_corner<C, T, 3, R>(cx, ldb); break;
+                    case 4: tile_corner<C, T, 4, R>(cx, ldb); break;
+                    case 5: tile_corner<C, T, 5, R>(cx, ldb); break;
+                    case 6: tile_corner<C, T, 6, R>(cx, ldb); break;
+                    case 7: tile_corner<C, T, 7, R>(cx, ldb); break;
+                    default: tile_corner<C, T, 8, R>(cx, ldb); break;
                 }
-                for (; e < e1; e += CPR) acc = fma(-slamv[e], ldb(s_lo + slamc[e]), acc);
-                acc += (a1 + a2) + a3;
+            } else if (k > 0) {
+                // k > 8 (rare): CSR spmv and getrs through shared memory
+                C *x1 = sx1 + (it & 1) * R * k + rr * k;
+                for (int d = 0; d < k; ++d) {
+                    C acc = part == 0 ? ldb(sdrow[d]) * sdscale[d] : C(0);
+                    for (int e = slamptr[d] + part; e < slamptr[d + 1]; e += CPR)
+                        acc = fma(-slamv[e], ldb(s_lo + slamc[e]), acc);
 #pragma unroll
-                for (int off = R; off < 32; off *= 2) acc += __shfl_xor_sync(0xffffffffu, acc, off);
-                if (part == 0) x1[d] = acc;
-            }
-            SB_TR(3);
-            if (part == 0 && k > 0) {
-                getrs_small(x1, sdlu, sdpiv, k);
-                if (clive)
-                    for (int d = 0; d < k; ++d) __stcs(gs + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
+                    for (int off = R; off < 32; off *= 2) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+                    if (part == 0) x1[d] = acc;
+                }
+                SB_TR(3);
+                if (part == 0) {
+                    getrs_small(x1, sdlu, sdpiv, k);
+                    if (clive)
+                        for (int d = 0; d < k; ++d) __stcs(gs + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
+                }
+                __syncwarp();
+                if (cx.patch) patch_gamma_smem<C, T, R>(cx, k);
             }
             SB_TR(1);
             __syncwarp();
@@ -605,9 +777,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const int a = s * L;
     const bool full_seg = a + L <= nQ;
     const int sc = G.slot[active ? s : 0];  // factor block (idle threads alias segment 0)
-    const C *fL = sL + (size_t)sc * LP;
-    const C *fU = sU + (size_t)sc * LP;
-    const C *fD = sdinv + (size_t)sc * LP;
+    const C *fL = sF + sc * (2 * K + 1) * LP;  // one base register; bands at immediate offsets
+    const C *fU = fL + K * LP;
+    const C *fD = fL + 2 * K * LP;
     // boxes this warp reads (rows of its real segments)
     int c_lo = 0, c_hi = -1;
     {
@@ -619,7 +791,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             c_hi = rr1 / boxr;
         }
     }
-    const int nthr_c = ncw * 32;
+    // this warp owns gamma rows: it waits for the corner warp's patch of the tile
+    const bool wgam = __any_sync(0xffffffffu, active && sgptr[s] < sgptr[s + 1]);
     int it = 0;
     for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
         const int slab = tile / p.tps;
@@ -632,29 +805,19 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         // ---------- own segment of b0 into registers
         if (LOADER == LOAD_TMA) {
             for (int c = c_lo; c <= c_hi; ++c) mbar_wait(full + c, it & 1);
+            if (gpatch && wgam) mbar_wait(gready + (it & 1), (it >> 1) & 1);  // gamma rows patched by the corner warp
             SB_TR(8);
+            // one predicated path for full and partial segments (no divergence in the
+            // warp that holds the last, partial segment)
             const T *src = buf + (size_t)(s_lo + a) * R + r0;
-            if (full_seg) {
 #pragma unroll
-                for (int i = 0; i < L; ++i) {
-                    const V w = *reinterpret_cast<const V *>(src + (size_t)i * R);
-                    const T *pw = reinterpret_cast<const T *>(&w);
+            for (int i = 0; i < L; ++i) {
+                V w;
+                if (full_seg || (active && a + i < nQ)) w = *reinterpret_cast<const V *>(src + (size_t)i * R);
+                else w = V{};
+                const T *pw = reinterpret_cast<const T *>(&w);
 #pragma unroll
-                    for (int q = 0; q < NV; ++q) v[i][q] = (C)pw[q];
-                }
-            } else {
-#pragma unroll
-                for (int i = 0; i < L; ++i) {
-                    if (active && a + i < nQ) {
-                        const V w = *reinterpret_cast<const V *>(src + (size_t)i * R);
-                        const T *pw = reinterpret_cast<const T *>(&w);
-#pragma unroll
-                        for (int q = 0; q < NV; ++q) v[i][q] = (C)pw[q];
-                    } else {
-#pragma unroll
-                        for (int q = 0; q < NV; ++q) v[i][q] = C(0);
-                    }
-                }
+                for (int q = 0; q < NV; ++q) v[i][q] = (C)pw[q];
             }
             __syncwarp();
             if (lane == 0)
@@ -668,8 +831,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                     v[i][q] = (q < nlive && a + i < nQ) ? (C)__ldcs(src + (int64_t)i * ps + q * p.bstride) : C(0);
         }
         SB_TR(1);
-        // ---------- b0 -= gamma x1 (only segments holding gamma rows wait for the corner warp)
-        if (active && sgptr[s] < sgptr[s + 1]) {
+        // ---------- b0 -= gamma x1 unless the corner warp patched the tile in shared
+        // memory (only segments holding gamma rows wait for the corner warp)
+        if (!gpatch && active && sgptr[s] < sgptr[s + 1]) {
             mbar_wait(x1full + (it & 1), (it >> 1) & 1);
             const C *x1 = sx1 + (it & 1) * R * k + r0 * k;
             for (int e = sgptr[s]; e < sgptr[s + 1]; ++e) {
@@ -687,13 +851,14 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         // ---------- local forward sweep, publish end state
         C st[K][NV];
         fwd_local<C, K, L, NV, true>(v, fL, ms, st);
+        // end states in SoA order [j][segment][rhs]: consecutive lanes hit consecutive banks
         if (active)
 #pragma unroll
             for (int q = 0; q < NV; ++q)
 #pragma unroll
-                for (int j = 0; j < K; ++j) sfend[(s * R + r0 + q) * K + j] = st[j][q];
+                for (int j = 0; j < K; ++j) sfend[(j * S + s) * R + r0 + q] = st[j][q];
         SB_TR(3);
-        named_bar(1, nthr_c);  // B2
+        named_bar(1, ncw * 32);  // B2: every local forward end state is published
         SB_TR(4);
         // ---------- forward carry (true y at rows a-1..a-K) + correction chain
         if (active && s > 0) {
@@ -708,7 +873,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 for (int j = 0; j < K; ++j)
 #pragma unroll
                     for (int q = 0; q < NV; ++q) {
-                        C acc = sfend[(t * R + r0 + q) * K + j];
+                        C acc = sfend[(j * S + t) * R + r0 + q];
 #pragma unroll
                         for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m][q], acc);
                         nw[j][q] = acc;
@@ -726,9 +891,9 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
 #pragma unroll
             for (int q = 0; q < NV; ++q)
 #pragma unroll
-                for (int j = 0; j < K; ++j) sbbeg[(s * R + r0 + q) * K + j] = st[j][q];
+                for (int j = 0; j < K; ++j) sbbeg[(j * S + s) * R + r0 + q] = st[j][q];
         SB_TR(5);
-        named_bar(1, nthr_c);  // B3
+        named_bar(1, ncw * 32);  // B3: every local backward begin state is published
         SB_TR(6);
         // ---------- backward carry (true x at rows a+L..a+L+K-1) + correction chain
         // TMA path, band K >= 2: every row is stored from inside the chain as soon as
@@ -749,7 +914,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 for (int j = 0; j < K; ++j)
 #pragma unroll
                     for (int q = 0; q < NV; ++q) {
-                        C acc = sbbeg[(t * R + r0 + q) * K + j];
+                        C acc = sbbeg[(j * S + t) * R + r0 + q];
 #pragma unroll
                         for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m][q], acc);
                         nw[j][q] = acc;
@@ -759,10 +924,13 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
 #pragma unroll
                     for (int q = 0; q < NV; ++q) co[j][q] = nw[j][q];
             }
-            if constexpr (FUSED)
-                bwd_correct<C, K, L, NV, true, true, T>(v, fU, ms, co, gcol + (int64_t)(s_lo + a) * ps, ps,
-                                                        nlive > 0 ? min(L, nQ - a) : 0);
-            else
+            if constexpr (FUSED) {
+                // one code path for every segment (a full and the partial last segment
+                // share warp 13: two instantiations would run one after the other)
+                T *dlast = gcol + (int64_t)(s_lo + a + L - 1) * ps;
+                const int nvalid = nlive > 0 ? min(L, nQ - a) : 0;
+                bwd_correct<C, K, L, NV, true, true, true, T>(v, fU, ms, co, dlast, ps, nvalid);
+            } else
                 bwd_correct<C, K, L, NV, true>(v, fU, ms, co);
         }
         // ---------- store x0 straight from registers (one 16-B vector per row).
@@ -770,22 +938,27 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         // overwritten before x1 is done.
         if (LOADER == LOAD_DIRECT && k > 0) mbar_wait(x1full + (it & 1), (it >> 1) & 1);
         if (!FUSED && nlive > 0) {
+            // one predicated path for full and partial segments (no divergence in the
+            // warp that holds the last, partial segment); running row pointer
             T *dst = gcol + (int64_t)(s_lo + a) * ps;
-            if (LOADER == LOAD_TMA && nlive == NV && full_seg) {
+            if (LOADER == LOAD_TMA && nlive == NV) {
 #pragma unroll
                 for (int i = 0; i < L; ++i) {
                     V w;
                     T *pw = reinterpret_cast<T *>(&w);
 #pragma unroll
                     for (int q = 0; q < NV; ++q) pw[q] = (T)v[i][q];
-                    __stcs(reinterpret_cast<V *>(dst + (int64_t)i * ps), w);
+                    if (full_seg || a + i < nQ) __stcs(reinterpret_cast<V *>(dst), w);
+                    dst += ps;
                 }
             } else {
 #pragma unroll
-                for (int i = 0; i < L; ++i)
+                for (int i = 0; i < L; ++i) {
 #pragma unroll
                     for (int q = 0; q < NV; ++q)
-                        if (q < nlive && a + i < nQ) __stcs(dst + (int64_t)i * ps + q * p.bstride, (T)v[i][q]);
+                        if (q < nlive && a + i < nQ) __stcs(dst + q * p.bstride, (T)v[i][q]);
+                    dst += ps;
+                }
             }
         }
         SB_TR(7);
@@ -802,24 +975,6 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
 // one cp.async.bulk (global->smem, mbarrier complete_tx) into one of two
 // per-warp row buffers, so the next row streams in while this one is solved,
 // and writes the result back with one bulk smem->global copy.
-__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *mbar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                     smem_u32(dst)),
-                 "l"(src), "r"(bytes), "r"(smem_u32(mbar))
-                 : "memory");
-}
-__device__ __forceinline__ void bulk_store(void *dst, const void *src, uint32_t bytes) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
-                 "r"(bytes)
-                 : "memory");
-    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async_smem() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-
 // Algorithm 2's interpolation at the feet of the characteristics (PAPER.md
 // P:157-163): out[i] = S(xi_i - shift) for the periodic spline S with
 // coefficients coef[0..N) just solved for.  The p+1 nonzero B-splines at a
@@ -972,8 +1127,9 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
     const DevPlan &P = p.P;
     const DevSeg &G = P.seg[2];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int S = G.S, LP = G.LP, nQ = P.nQ, k = P.k, s_lo = P.s_lo, n = P.n;
-    const int ms = G.nslots * LP;
+    const int S = G.S, nQ = P.nQ, k = P.k, s_lo = P.s_lo, n = P.n;
+    constexpr int LP = L;  // odd factor pitch (conflict-free across the 32 lanes' segments)
+    constexpr int ms = LP;
     const int nwarps = blockDim.x >> 5;
 
     uint64_t *wbar = reinterpret_cast<uint64_t *>(smem + p.off_mbar) + 2 * warp;  // 2 per warp
@@ -993,9 +1149,7 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
     __syncthreads();
     mbar_wait(cbar, 0);
 
-    const C *sL = reinterpret_cast<const C *>(smem + p.off_L);
-    const C *sU = reinterpret_cast<const C *>(smem + p.off_U);
-    const C *sdinv = reinterpret_cast<const C *>(smem + p.off_dinv);
+    const C *sF = reinterpret_cast<const C *>(smem + p.off_L);
     const C *sG = reinterpret_cast<const C *>(smem + p.off_G);
     const C *sH = reinterpret_cast<const C *>(smem + p.off_H);
     const int *slamptr = reinterpret_cast<const int *>(smem + p.off_lamptr);
@@ -1016,9 +1170,9 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
     const bool active = s < S;
     const int a = s * L;
     const int slot = G.slot[active ? s : 0];  // identical segments share (and broadcast) one block
-    const C *fL = sL + (size_t)slot * LP;
-    const C *fU = sU + (size_t)slot * LP;
-    const C *fD = sdinv + (size_t)slot * LP;
+    const C *fL = sF + slot * (2 * K + 1) * LP;
+    const C *fU = fL + K * LP;
+    const C *fD = fL + 2 * K * LP;
     T *gout = reinterpret_cast<T *>(p.rhs);
     const int64_t ps = p.pstride;
     const bool vec = (ps == 1) && ((p.bstride * (int64_t)sizeof(T)) % 16 == 0) &&

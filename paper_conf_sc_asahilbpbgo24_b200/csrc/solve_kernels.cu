@@ -53,9 +53,8 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     };
     const int K = P.K, k = P.k, S = G.S;
     kp.off_buf = take(buf_bytes, 1024);
-    kp.off_L = take((size_t)K * G.nslots * G.LP * esz, 16);
-    kp.off_U = take((size_t)K * G.nslots * G.LP * esz, 16);
-    kp.off_dinv = take((size_t)G.nslots * G.LP * esz, 16);
+    kp.off_L = take((size_t)(2 * K + 1) * G.nslots * G.LP * esz, 16);  // factor blocks (DevSeg::F)
+    kp.off_U = kp.off_dinv = kp.off_L;
     kp.off_G = take((size_t)S * K * K * esz, 16);
     kp.off_H = take((size_t)S * K * K * esz, 16);
     kp.off_fend = take((size_t)S * R * K * esz, 16);
@@ -64,6 +63,9 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_lamptr = take((size_t)(k + 1) * 4, 16);
     kp.off_lamc = take((size_t)P.lam_nnz * 4, 16);
     kp.off_lamv = take((size_t)P.lam_nnz * esz, 16);
+    kp.off_lw = take((size_t)(P.lw_head + P.lw_tail) * k * esz, 16);
+    kp.off_grr = take((size_t)P.gr_n * 4, 16);
+    kp.off_grv = take((size_t)P.gr_n * k * esz, 16);
     kp.off_gamr = take((size_t)P.gam_nnz * 4, 16);
     kp.off_gamc = take((size_t)P.gam_nnz * 4, 16);
     kp.off_gamv = take((size_t)P.gam_nnz * esz, 16);
@@ -74,7 +76,8 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_drow = take((size_t)k * 4, 16);
     kp.off_cbuf = take((size_t)4 * cbox * R * esz, 128);
     kp.off_geo = take(geo_bytes, 16);
-    kp.off_mbar = take((size_t)std::max(2 * NBOXMAX + 5, 2 * WARP_MAX_WARPS + 1) * 8, 8);  // tile: boxes; warp: 2 per warp; + constants
+    // tile: full/empty per box, x1full[2], cfull[3]; warp kernel: 2 per warp + constants
+    kp.off_mbar = take((size_t)std::max(2 * NBOXMAX + 7, 2 * WARP_MAX_WARPS + 1) * 8, 8);
     kp.smem_total = (int)align_up(o, 16);
     return kp.smem_total;
 }
@@ -222,6 +225,10 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     }
     const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
     const int L = G.L;
+    if (G.LP != L + (esz == 8 ? 2 : 4)) {  // the tile kernel's compile-time factor pitch
+        snprintf(err, errlen, "tile plan pitch %d does not match L=%d", G.LP, L);
+        return 5;
+    }
     KParams kp{};
     kp.P = P;
     kp.rhs = a.rhs;
@@ -305,6 +312,16 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     }
     for (int c = 0; c < NBOXMAX; ++c)
         if (kp.empty_count[c] == 0) kp.empty_count[c] = 1;  // unused boxes: any valid count
+    // boxes holding gamma rows: the corner warp waits for them before patching
+    kp.gbox_mask = 0;
+    if (loader == LOAD_TMA && P.gam_nnz > 0) {
+        if (P.gam_head > 0)
+            for (int c = P.s_lo / boxr; c <= (P.s_lo + P.gam_head - 1) / boxr; ++c) kp.gbox_mask |= 1 << c;
+        if (P.gam_tail > 0)
+            for (int c = (P.s_lo + P.nQ - P.gam_tail) / boxr; c <= (P.s_lo + P.nQ - 1) / boxr; ++c)
+                kp.gbox_mask |= 1 << c;
+    }
+
     CUtensorMap tm[2];
     memset(tm, 0, sizeof(tm));
     if (loader == LOAD_TMA) {
