@@ -517,6 +517,8 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     for _ in range(args.warmup):
         step(x)
+    from paper_conf_sc_asahilbpbgo24_b200 import last_kernel
+    kernel_name = last_kernel()
     barrier()
     run_chunk = ChunkRunner(lambda: step(x), not args.no_graph)
     nchunks = (args.steps + CHUNK - 1) // CHUNK
@@ -612,7 +614,9 @@ def main():
                        "l2": f"inputs {n * B * esz / 1e6:.0f} MB per GPU > 126 MB L2; input restored + 256 MB "
                              f"L2 flush every 40 steps (untimed)",
                        "inputs": "device Philox (inputs.rhs_device)" if on_device else "host Philox (inputs.rhs)",
-                       "launch": "python per step" if args.no_graph else "CUDA graph of 40 launches, replayed",
+                       "launch": "python per step" if args.no_graph else
+                       f"CUDA graphs of up to {CHUNK} launches, replayed",
+                       "kernel": kernel_name,
                        "parallelism": f"dp{ws} (RHS shards)"},
             "ms_per_step_median": float(np.median(per_chunk)), "ms_per_step_best": float(min(per_chunk)),
             "timed_chunks": len(per_chunk),

@@ -466,6 +466,8 @@ template <typename C, typename T> struct CornerCtx {
     C *sx1;       // this lane's x1 slot (DIRECT loader / k > 8)
     T *gout;      // column of this RHS in HBM (nullptr: RHS beyond the batch)
     int64_t ps;
+    const T *hb, *tb;  // b at the first row of the Lambda window's head / tail (this RHS)
+    int64_t bst;       // elements between consecutive rows there
     bool patch;   // gamma patched into the shared-memory tile by this warp (else x1 -> sx1)
 };
 
@@ -532,24 +534,28 @@ __device__ __forceinline__ void tile_corner(const CornerCtx<C, T> &cx, LDB ldb) 
     C xr[KC];
 #pragma unroll
     for (int d = 0; d < KC; ++d) xr[d] = C(0);
+    // the window's head columns are rows hb[j*bst], its tail columns rows tb[j*bst]
+    // (j from 0): batches of JB columns per lane with immediate offsets, the b
+    // loads and the Lambda loads of a batch independent of each other
     constexpr int JB = 8;
-    for (int j0 = cx.part; j0 < cx.lw; j0 += JB * CPR) {
-        C b[JB];
+    auto window = [&](const T *base, const C *lv, int len) {
+        base += (int64_t)cx.part * cx.bst;
+        lv += cx.part * KC;
+        for (int j0 = cx.part; j0 < len; j0 += JB * CPR) {
+            C b[JB];
 #pragma unroll
-        for (int u = 0; u < JB; ++u) {
-            const int j = j0 + u * CPR;
-            b[u] = j < cx.lw ? ldb(j < cx.lh ? cx.s_lo + j : cx.tail0 + j) : C(0);
+            for (int u = 0; u < JB; ++u) b[u] = j0 + u * CPR < len ? (C)base[(int64_t)u * CPR * cx.bst] : C(0);
+#pragma unroll
+            for (int u = 0; u < JB; ++u)
+                if (j0 + u * CPR < len)
+#pragma unroll
+                    for (int d = 0; d < KC; ++d) xr[d] = fma(-lv[u * CPR * KC + d], b[u], xr[d]);
+            base += (int64_t)JB * CPR * cx.bst;
+            lv += JB * CPR * KC;
         }
-#pragma unroll
-        for (int u = 0; u < JB; ++u) {
-            const int j = j0 + u * CPR;
-            if (j < cx.lw) {
-                const C *lv = cx.slw + j * KC;
-#pragma unroll
-                for (int d = 0; d < KC; ++d) xr[d] = fma(-lv[d], b[u], xr[d]);
-            }
-        }
-    }
+    };
+    window(cx.hb, cx.slw, cx.lh);
+    window(cx.tb, cx.slw + cx.lh * KC, cx.lw - cx.lh);
 #pragma unroll
     for (int d = 0; d < KC; ++d) {
         C acc = xr[d];
@@ -723,6 +729,23 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             cx.sx1 = sx1 + (it & 1) * R * k + rr * k;
             cx.gout = clive ? gs + ccol * p.bstride : nullptr; cx.ps = ps;
             cx.patch = gpatch;
+            {   // where the window rows of this RHS live: corner boxes, main tile or HBM
+                const int hr = s_lo, tr = s_lo + nQ - P.lw_tail;  // first rows of head / tail windows
+                if (LOADER == LOAD_TMA) {
+                    cx.bst = R;
+                    if (use_cbox) {
+                        cx.hb = cb + (size_t)hr * R + rr;
+                        cx.tb = cb + (size_t)(cbox + tr - (P.n - cbox)) * R + rr;
+                    } else {
+                        cx.hb = buf + (size_t)hr * R + rr;
+                        cx.tb = buf + (size_t)tr * R + rr;
+                    }
+                } else {
+                    cx.bst = clive ? ps : 0;  // beyond the batch: read row 0 of column 0, times 0
+                    cx.hb = clive ? ccolp + (int64_t)hr * ps : gout;
+                    cx.tb = clive ? ccolp + (int64_t)tr * ps : gout;
+                }
+            }
             if (k >= 1 && k <= WCORNER_KREG) {
                 // x1 in registers with k a compile-time constant (every instruction of the
                 // corner warp costs ~4 issue cycles next to the compute warps)
