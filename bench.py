@@ -456,6 +456,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-graph", action="store_true", help="launch each step from Python instead of a CUDA graph")
+    ap.add_argument("--split", default=None, help="force the Schur split LO,HI (default: chosen at create)")
     args = ap.parse_args()
     if args.workload in TWOD:
         if args.impl == "reference":
@@ -481,7 +482,8 @@ def main():
     B_total = Bspec if strong else ws * Bspec
     n = inputs.nbasis(deg, npts, bc)
     knots = inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh)
-    sb = SplineBuilder(deg, npts, bc, knots)
+    split = tuple(int(v) for v in args.split.split(",")) if args.split else None
+    sb = SplineBuilder(deg, npts, bc, knots, split=split)
     esz = 4 if dt == "f32" else 8
     tdt = torch.float32 if dt == "f32" else torch.float64
     on_device = n * B > DEVICE_INPUT_ELEMS and layout == "batch"
@@ -616,7 +618,7 @@ def main():
                        "inputs": "device Philox (inputs.rhs_device)" if on_device else "host Philox (inputs.rhs)",
                        "launch": "python per step" if args.no_graph else
                        f"CUDA graphs of up to {CHUNK} launches, replayed",
-                       "kernel": kernel_name,
+                       "kernel": kernel_name, "split": [sb.info()["split_lo"], sb.info()["split_hi"]],
                        "parallelism": f"dp{ws} (RHS shards)"},
             "ms_per_step_median": float(np.median(per_chunk)), "ms_per_step_best": float(min(per_chunk)),
             "timed_chunks": len(per_chunk),

@@ -165,17 +165,7 @@ int upload(spline_builder *h) {
             const int j = c < lw_head ? c : lw_head + (c - (nQ - lw_tail));
             lw_v[(size_t)j * k + d] = P.Lam_v[e];
         }
-    std::vector<int> gr_row;
-    std::vector<double> gr_v;
-    for (size_t e = 0; e < P.gam_r.size(); ++e) {
-        if (gr_row.empty() || gr_row.back() != P.gam_r[e]) {
-            gr_row.push_back(P.gam_r[e]);
-            gr_v.resize(gr_v.size() + k, 0.0);
-        }
-        gr_v[(gr_row.size() - 1) * k + P.gam_c[e]] += P.gam_v[e];
-    }
     size_t o_lw[2] = {pk.addv(lw_v), pk.addv(conv<float>(lw_v))};
-    size_t o_grr = pk.addv(gr_row), o_grv[2] = {pk.addv(gr_v), pk.addv(conv<float>(gr_v))};
     size_t o_lamptr = pk.addv(P.Lam_ptr), o_lamc = pk.addv(P.Lam_c), o_gamr = pk.addv(P.gam_r),
            o_gamc = pk.addv(P.gam_c), o_dpiv = pk.addv(P.dpiv), o_drow = pk.addv(P.drow);
     h->blob_bytes = std::max<size_t>(pk.bytes.size(), 16);
@@ -201,11 +191,6 @@ int upload(spline_builder *h) {
         for (int r : P.drow) note(r);
         for (int c : P.Lam_c) note(P.s_lo + c);
         d.corner_rows = k > 0 ? std::max(head, tail) : 0;
-        d.gam_head = d.gam_tail = 0;
-        for (int r : P.gam_r) {
-            if (r < nQ / 2) d.gam_head = std::max(d.gam_head, r + 1);
-            else d.gam_tail = std::max(d.gam_tail, nQ - r);
-        }
     }
     for (int c = 0; c < 2; ++c) {
         d.lam_v[c] = at(oLam[c]); d.gam_v[c] = at(oGam[c]); d.dlu[c] = at(oDlu[c]); d.dscale[c] = at(oDs[c]);
@@ -228,9 +213,8 @@ int upload(spline_builder *h) {
     d.adv_tbl = (const int *)at(oTbl); d.adv_nbkt = (int)P.adv_tbl.size(); d.adv_steps = P.adv_steps;
     d.adv_bscale = P.xe.empty() ? 0.0 : (double)P.adv_tbl.size() / (P.xb[P.N] - P.xb[0]);
     d.lam_ptr = (const int *)at(o_lamptr); d.lam_c = (const int *)at(o_lamc);
-    d.lw_head = lw_head; d.lw_tail = lw_tail; d.gr_n = (int)gr_row.size();
-    d.gr_row = (const int *)at(o_grr);
-    for (int c = 0; c < 2; ++c) { d.lw_v[c] = at(o_lw[c]); d.gr_v[c] = at(o_grv[c]); }
+    d.lw_head = lw_head; d.lw_tail = lw_tail;
+    for (int c = 0; c < 2; ++c) d.lw_v[c] = at(o_lw[c]);
     d.gam_r = (const int *)at(o_gamr); d.gam_c = (const int *)at(o_gamc);
     d.dpiv = (const int *)at(o_dpiv); d.drow = (const int *)at(o_drow);
     return 0;

@@ -31,7 +31,6 @@ struct DevPlan {
     int n, nQ, s_lo, k, K;   // order, Q order, Q offset, delta order, kernel band
     int lam_nnz, gam_nnz;    // Lambda CSR / gamma COO sizes
     int corner_rows;         // rows [0,c) and [n-c,n) hold every row the corner reads (0: none/unbounded)
-    int gam_head, gam_tail;  // gamma rows lie in Q rows [0, gam_head) and [nQ-gam_tail, nQ)
     const void *lam_v[2], *gam_v[2], *dlu[2], *dscale[2];
     const void *rowf[2];     // nQ x (2K+1): L(i,i-1..i-K), U'(i,i+1..i+K), dinv(i) -- serial fallback
     int p, N, periodic;      // spline degree, cells, periodic flag (advection / evaluation)
@@ -43,14 +42,12 @@ struct DevPlan {
     int adv_nbkt, adv_steps;
     double adv_bscale;       // adv_nbkt / (x_N - x_0)
     const int *lam_ptr, *lam_c, *gam_r, *gam_c, *dpiv, *drow;
-    // Tile-kernel corner (dense, so every shared-memory load is independent of
-    // the others -- no column-index load in front of each b load):
-    //   Lambda on a column window: Q columns [0, lw_head) then [nQ-lw_tail, nQ),
-    //   lw_v[j*k + d] = Lambda(d, column j of the window) (0 where dropped);
-    //   gamma by distinct row: Q row gr_row[g], gr_v[g*k + d] = gamma(row, d).
-    int lw_head, lw_tail, gr_n;
-    const void *lw_v[2], *gr_v[2];
-    const int *gr_row;
+    // Tile-kernel corner: Lambda on a dense column window, Q columns [0, lw_head)
+    // then [nQ-lw_tail, nQ); lw_v[j*k + d] = Lambda(d, column j of the window)
+    // (0 where dropped), so every shared-memory load of the spmv is independent
+    // of the others (no column-index load in front of each b load)
+    int lw_head, lw_tail;
+    const void *lw_v[2];
     DevSeg seg[3];           // [0] tile kernel fp64 (L=36), [1] tile kernel fp32 (L=72),
                              // [2] warp-per-RHS kernel (odd L; S == 0 if unavailable)
 };

@@ -77,8 +77,7 @@ struct KParams {
     int corner_arrive_mask;          // boxes without a compute-warp reader: the corner warp frees them
     int cbox;                        // rows of each corner box (0: corner reads the main tile)
     // dynamic shared memory offsets (bytes)
-    int off_lw, off_grr, off_grv;    // tile corner: Lambda window, gamma rows (DevPlan::lw_*, gr_*)
-    int gbox_mask;                   // tile kernel: TMA boxes holding gamma rows (the corner warp patches them)
+    int off_lw;                      // tile corner: Lambda window (DevPlan::lw_*)
     int off_buf, off_L, off_U, off_dinv, off_G, off_H, off_fend, off_bbeg, off_x1, off_lamptr, off_lamc, off_lamv,
         off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, off_cbuf,
         smem_total;
@@ -414,8 +413,6 @@ __device__ __forceinline__ void stage_constants_issue(const KParams &p, const De
     stage_one(smem + p.off_lamc, P.lam_c, (size_t)P.lam_nnz * 4, cbar);
     stage_one(smem + p.off_lamv, P.lam_v[CI], (size_t)P.lam_nnz * esz, cbar);
     stage_one(smem + p.off_lw, P.lw_v[CI], (size_t)(P.lw_head + P.lw_tail) * k * esz, cbar);
-    stage_one(smem + p.off_grr, P.gr_row, (size_t)P.gr_n * 4, cbar);
-    stage_one(smem + p.off_grv, P.gr_v[CI], (size_t)P.gr_n * k * esz, cbar);
     stage_one(smem + p.off_gamr, P.gam_r, (size_t)P.gam_nnz * 4, cbar);
     stage_one(smem + p.off_gamc, P.gam_c, (size_t)P.gam_nnz * 4, cbar);
     stage_one(smem + p.off_gamv, P.gam_v[CI], (size_t)P.gam_nnz * esz, cbar);
@@ -458,76 +455,20 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // x1 = delta'^{-1} (s1 b1 - Lambda b0) for one tile (one RHS per lane pair),
 // run by the corner/producer warp one tile ahead of the compute warps.
 template <typename C, typename T> struct CornerCtx {
-    int part, rr, s_lo, it, nbox, gbox_mask, lh, lw, tail0, gr_n;
-    const C *slw, *sgrv, *sdlu, *sdscale;
-    const int *sgrr, *sdrow, *sdpiv;
-    uint64_t *full, *gready;
-    T *buf;
-    C *sx1;       // this lane's x1 slot (DIRECT loader / k > 8)
-    T *gout;      // column of this RHS in HBM (nullptr: RHS beyond the batch)
+    int part, lh, lw;
+    const C *slw, *sdlu, *sdscale;
+    const int *sdrow, *sdpiv;
+    C *sx1;            // this lane's x1 slot in shared memory
+    T *gout;           // column of this RHS in HBM (nullptr: RHS beyond the batch)
     int64_t ps;
     const T *hb, *tb;  // b at the first row of the Lambda window's head / tail (this RHS)
     int64_t bst;       // elements between consecutive rows there
-    bool patch;   // gamma patched into the shared-memory tile by this warp (else x1 -> sx1)
 };
-
-// TMA path: the corner warp applies b0 -= gamma x1 to the gamma rows of the
-// tile in the shared-memory boxes once they have landed, so the compute warps
-// neither wait for x1 nor select rows by a runtime index.  All loads first,
-// then all stores; then the generic->async proxy fence (the boxes are refilled
-// by TMA later) and the arrival on gready.
-template <typename C, typename T, int R>
-__device__ __forceinline__ void patch_gamma_done(const CornerCtx<C, T> &cx) {
-    fence_proxy_async_smem();
-    __syncwarp();
-    if (cx.part == 0) mbar_arrive(cx.gready + (cx.it & 1));
-}
-template <typename C, typename T, int R>
-__device__ __forceinline__ void patch_gamma_wait(const CornerCtx<C, T> &cx) {
-    for (int c = 0; c < cx.nbox; ++c)
-        if ((cx.gbox_mask >> c) & 1) mbar_wait(cx.full + c, cx.it & 1);
-}
-template <typename C, typename T, int R, int KC>
-__device__ __forceinline__ void patch_gamma_reg(const CornerCtx<C, T> &cx, const C (&xr)[KC]) {
-    patch_gamma_wait<C, T, R>(cx);
-    if (cx.part == 0) {
-        constexpr int GB = 8;
-        for (int g0 = 0; g0 < cx.gr_n; g0 += GB) {
-            int off[GB];
-            C val[GB];
-#pragma unroll
-            for (int g = 0; g < GB; ++g) {
-                off[g] = g0 + g < cx.gr_n ? (cx.s_lo + cx.sgrr[g0 + g]) * R + cx.rr : -1;
-                val[g] = off[g] >= 0 ? (C)cx.buf[off[g]] : C(0);
-            }
-#pragma unroll
-            for (int g = 0; g < GB; ++g) {
-                C acc = val[g];
-#pragma unroll
-                for (int d = 0; d < KC; ++d) acc = fma(-cx.sgrv[(g0 + g) * KC + d], xr[d], acc);
-                if (off[g] >= 0) cx.buf[off[g]] = (T)acc;
-            }
-        }
-    }
-    patch_gamma_done<C, T, R>(cx);
-}
-template <typename C, typename T, int R>
-__device__ __forceinline__ void patch_gamma_smem(const CornerCtx<C, T> &cx, int k) {
-    patch_gamma_wait<C, T, R>(cx);
-    if (cx.part == 0)
-        for (int g = 0; g < cx.gr_n; ++g) {
-            T *q = cx.buf + (cx.s_lo + cx.sgrr[g]) * R + cx.rr;
-            C acc = (C)*q;
-            for (int d = 0; d < k; ++d) acc = fma(-cx.sgrv[g * k + d], cx.sx1[d], acc);
-            *q = (T)acc;
-        }
-    patch_gamma_done<C, T, R>(cx);
-}
 
 // k = KC <= 8: Lambda on its dense column window (each b row loaded once for
 // all KC rows; loads in independent batches), xor-shuffle over the CPR lanes
-// of a RHS, getrs on registers, delta rows of x to HBM, gamma patch (TMA) or
-// x1 to shared memory (DIRECT loader: the compute warps apply gamma).
+// of a RHS, getrs on registers, delta rows of x to HBM, x1 to shared memory
+// (the compute warps holding gamma rows apply b0 -= gamma x1).
 template <typename C, typename T, int KC, int R, typename LDB>
 __device__ __forceinline__ void tile_corner(const CornerCtx<C, T> &cx, LDB ldb) {
     constexpr int CPR = 32 / R;
@@ -567,9 +508,7 @@ __device__ __forceinline__ void tile_corner(const CornerCtx<C, T> &cx, LDB ldb) 
     if (cx.part == 0 && cx.gout)
 #pragma unroll
         for (int d = 0; d < KC; ++d) __stcs(cx.gout + (int64_t)cx.sdrow[d] * cx.ps, (T)xr[d]);
-    if (cx.patch) {
-        patch_gamma_reg<C, T, R, KC>(cx, xr);
-    } else if (cx.part == 0) {
+    if (cx.part == 0) {
 #pragma unroll
         for (int d = 0; d < KC; ++d) cx.sx1[d] = xr[d];
     }
@@ -623,8 +562,6 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     const int *slamc = reinterpret_cast<const int *>(smem + p.off_lamc);
     const C *slamv = reinterpret_cast<const C *>(smem + p.off_lamv);
     const C *slw = reinterpret_cast<const C *>(smem + p.off_lw);
-    const int *sgrr = reinterpret_cast<const int *>(smem + p.off_grr);
-    const C *sgrv = reinterpret_cast<const C *>(smem + p.off_grv);
     const int *sgamr = reinterpret_cast<const int *>(smem + p.off_gamr);
     const int *sgamc = reinterpret_cast<const int *>(smem + p.off_gamc);
     const C *sgamv = reinterpret_cast<const C *>(smem + p.off_gamv);
@@ -637,15 +574,10 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
     uint64_t *empty = full + NBOXMAX;
     uint64_t *x1full = empty + NBOXMAX;
     uint64_t *cfull = x1full + 2;  // corner boxes, double-buffered (+ [2]: constants staged)
-    uint64_t *gready = cfull + 3;  // TMA path: gamma rows of the tile patched in smem, double-buffered
     T *buf = reinterpret_cast<T *>(smem + p.off_buf);
     T *cbuf = reinterpret_cast<T *>(smem + p.off_cbuf);  // [2][2 boxes][cbox rows][R]
     const int cbox = p.cbox;
     const bool use_cbox = LOADER == LOAD_TMA && cbox > 0;
-    // gamma patched in shared memory by the corner warp: only when x1 is computed a
-    // tile ahead from the corner boxes (without them the gamma warps would wait for
-    // x1 before they even load their rows)
-    const bool gpatch = use_cbox;
     T *gout = reinterpret_cast<T *>(p.rhs);
     const int64_t ps = p.pstride;
     const uint32_t box_bytes = (uint32_t)(boxr * R * sizeof(T));
@@ -660,8 +592,6 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         mbar_init(cfull + 0, 1);
         mbar_init(cfull + 1, 1);
         mbar_init(cfull + 2, 1);  // constants staged
-        mbar_init(gready + 0, R);  // every patching corner lane arrives
-        mbar_init(gready + 1, R);
         fence_mbar_init();
         if (LOADER == LOAD_TMA) prefetch_tmap(&tmap);
         if (use_cbox) prefetch_tmap(&tmap_c);
@@ -722,13 +652,10 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 return clive ? (C)ccolp[(int64_t)row * ps] : C(0);
             };
             CornerCtx<C, T> cx;
-            cx.part = part; cx.rr = rr; cx.s_lo = s_lo; cx.it = it; cx.nbox = nbox; cx.gbox_mask = p.gbox_mask;
-            cx.lh = P.lw_head; cx.lw = P.lw_head + P.lw_tail; cx.tail0 = s_lo + nQ - P.lw_tail - P.lw_head;
-            cx.gr_n = P.gr_n; cx.slw = slw; cx.sgrv = sgrv; cx.sdlu = sdlu; cx.sdscale = sdscale;
-            cx.sgrr = sgrr; cx.sdrow = sdrow; cx.sdpiv = sdpiv; cx.full = full; cx.gready = gready; cx.buf = buf;
+            cx.part = part; cx.lh = P.lw_head; cx.lw = P.lw_head + P.lw_tail;
+            cx.slw = slw; cx.sdlu = sdlu; cx.sdscale = sdscale; cx.sdrow = sdrow; cx.sdpiv = sdpiv;
             cx.sx1 = sx1 + (it & 1) * R * k + rr * k;
             cx.gout = clive ? gs + ccol * p.bstride : nullptr; cx.ps = ps;
-            cx.patch = gpatch;
             {   // where the window rows of this RHS live: corner boxes, main tile or HBM
                 const int hr = s_lo, tr = s_lo + nQ - P.lw_tail;  // first rows of head / tail windows
                 if (LOADER == LOAD_TMA) {
@@ -776,8 +703,6 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                     if (clive)
                         for (int d = 0; d < k; ++d) __stcs(gs + ccol * p.bstride + (int64_t)sdrow[d] * ps, (T)x1[d]);
                 }
-                __syncwarp();
-                if (cx.patch) patch_gamma_smem<C, T, R>(cx, k);
             }
             SB_TR(1);
             __syncwarp();
@@ -814,8 +739,6 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             c_hi = rr1 / boxr;
         }
     }
-    // this warp owns gamma rows: it waits for the corner warp's patch of the tile
-    const bool wgam = __any_sync(0xffffffffu, active && sgptr[s] < sgptr[s + 1]);
     int it = 0;
     for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x, ++it) {
         const int slab = tile / p.tps;
@@ -828,7 +751,6 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         // ---------- own segment of b0 into registers
         if (LOADER == LOAD_TMA) {
             for (int c = c_lo; c <= c_hi; ++c) mbar_wait(full + c, it & 1);
-            if (gpatch && wgam) mbar_wait(gready + (it & 1), (it >> 1) & 1);  // gamma rows patched by the corner warp
             SB_TR(8);
             // one predicated path for full and partial segments (no divergence in the
             // warp that holds the last, partial segment)
@@ -854,9 +776,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                     v[i][q] = (q < nlive && a + i < nQ) ? (C)__ldcs(src + (int64_t)i * ps + q * p.bstride) : C(0);
         }
         SB_TR(1);
-        // ---------- b0 -= gamma x1 unless the corner warp patched the tile in shared
-        // memory (only segments holding gamma rows wait for the corner warp)
-        if (!gpatch && active && sgptr[s] < sgptr[s + 1]) {
+        // ---------- b0 -= gamma x1 (only segments holding gamma rows wait for the corner warp)
+        if (active && sgptr[s] < sgptr[s + 1]) {
             mbar_wait(x1full + (it & 1), (it >> 1) & 1);
             const C *x1 = sx1 + (it & 1) * R * k + r0 * k;
             for (int e = sgptr[s]; e < sgptr[s + 1]; ++e) {

@@ -64,8 +64,6 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_lamc = take((size_t)P.lam_nnz * 4, 16);
     kp.off_lamv = take((size_t)P.lam_nnz * esz, 16);
     kp.off_lw = take((size_t)(P.lw_head + P.lw_tail) * k * esz, 16);
-    kp.off_grr = take((size_t)P.gr_n * 4, 16);
-    kp.off_grv = take((size_t)P.gr_n * k * esz, 16);
     kp.off_gamr = take((size_t)P.gam_nnz * 4, 16);
     kp.off_gamc = take((size_t)P.gam_nnz * 4, 16);
     kp.off_gamv = take((size_t)P.gam_nnz * esz, 16);
@@ -271,9 +269,14 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     // corner boxes: the corner reads only rows [0,cbox) and [n-cbox,n); they are
     // fetched one tile early with their own (smaller) tensor map
     int cbox = 0;
-    static const int cbox_env = [] {  // SB_TILE_CBOX=0 disables corner boxes (A/B experiments)
+    // Off by default since the corner became a k-templated register computation on
+    // hardware warp 0 reading a dense Lambda window: it now finishes from the landed
+    // tile in time, and the corner boxes only cost shared memory and L2 re-reads
+    // (measured: C3 Hermite 0.298 ms with them, 0.276 ms without; C2, C3 Greville,
+    // C4M unchanged).  SB_TILE_CBOX=1 enables them where they fit (A/B experiments).
+    static const int cbox_env = [] {
         const char *e = getenv("SB_TILE_CBOX");
-        return e ? atoi(e) : 1;
+        return e ? atoi(e) : 0;
     }();
     // worth it only when the corner step is heavy enough to delay the gamma warps
     // (measured: k=1 / 48 nnz C2 loses 4.6 %, k=6 Hermite C3 gains 16 %)
@@ -312,16 +315,6 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     }
     for (int c = 0; c < NBOXMAX; ++c)
         if (kp.empty_count[c] == 0) kp.empty_count[c] = 1;  // unused boxes: any valid count
-    // boxes holding gamma rows: the corner warp waits for them before patching
-    kp.gbox_mask = 0;
-    if (loader == LOAD_TMA && P.gam_nnz > 0) {
-        if (P.gam_head > 0)
-            for (int c = P.s_lo / boxr; c <= (P.s_lo + P.gam_head - 1) / boxr; ++c) kp.gbox_mask |= 1 << c;
-        if (P.gam_tail > 0)
-            for (int c = (P.s_lo + P.nQ - P.gam_tail) / boxr; c <= (P.s_lo + P.nQ - 1) / boxr; ++c)
-                kp.gbox_mask |= 1 << c;
-    }
-
     CUtensorMap tm[2];
     memset(tm, 0, sizeof(tm));
     if (loader == LOAD_TMA) {
