@@ -47,8 +47,12 @@ enum {
 };
 /* create flags */
 enum {
-    SB_FLAG_HOST_ONLY = 1 /* factor on the host only; no device upload (solve_* then
-                             return SB_UNSUPPORTED).  For inspection / CPU tests. */
+    SB_FLAG_HOST_ONLY = 1,    /* factor on the host only; no device upload (solve_* then
+                                 return SB_UNSUPPORTED).  For inspection / CPU tests. */
+    SB_FLAG_DEVICE_UPDATE = 2 /* structure frozen for spline_builder_update_device: the
+                                 gamma / Lambda patterns are dilated by 24 rows / columns,
+                                 segment carries one deeper, no factor sharing between
+                                 segments (uniform meshes solve slightly slower) */
 };
 
 /*
@@ -110,6 +114,37 @@ spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, cons
  * matrix).  Re-capture graphs after an update to solve with the new mesh.
  * Each host update retires one blob (~10-200 KB) until destroy. */
 int spline_builder_update(spline_builder_t h, const double *knots);
+
+/*
+ * spline_builder_update_device -- new mesh, factorised ON THE DEVICE (SURVEY
+ * 8(f)4; BASELINE north_star "one-time host or device factorisation"), for a
+ * handle created with SB_FLAG_DEVICE_UPDATE.  One kernel on `stream`
+ * recomputes, for the breakpoints `knots` (DEVICE pointer, N+1 strictly
+ * increasing values, read by the kernel; NULL = uniform on [0,1]), the
+ * collocation matrix (de Boor BSPLVB/BSPLVD), the Schur blocks of Eq. 3
+ * (P:69-78), the banded LU of Q without interchanges (Table I), beta = Q^-1 gamma,
+ * Lambda = lambda Q^-1, delta' = delta - lambda beta and its LU (Eq. 4-6), and
+ * every layout the solve kernels read, into a staging copy of the handle's
+ * device constants; the copy replaces the live constants in stream order only
+ * if every check passed.  Asynchronous: solves enqueued later on the same
+ * stream use the new mesh; solves on other streams must be ordered by the
+ * caller.  Kernels captured in a CUDA graph keep valid arguments and see the
+ * new mesh on replay.  Checks (reported by spline_builder_update_status, the
+ * previous mesh kept on failure): knots strictly increasing (SB_INVALID_ARG);
+ * a periodic mesh keeps its end points (SB_INVALID_ARG); Q / delta' factor
+ * without breakdown or growth > 1e3 (SB_SINGULAR); the new matrix fits the
+ * frozen band, gamma / Lambda (|Lambda| > 1e-14) patterns, carry depths and
+ * advection buckets (SB_UNSUPPORTED: re-plan with spline_builder_update).
+ * Host-side queries (get_info, get_blocks, solve_cpu_plan) keep describing the
+ * mesh of the last host create/update.  Returns SB_UNSUPPORTED for handles
+ * without the flag.
+ */
+int spline_builder_update_device(spline_builder_t h, const double *knots, void *stream);
+
+/* Waits for the last spline_builder_update_device on h and returns its
+ * outcome (SB_OK: the new mesh is live; else the previous mesh is kept and
+ * spline_builder_last_error() says why).  SB_OK if none is pending. */
+int spline_builder_update_status(spline_builder_t h);
 
 /*
  * spline_builder_solve -- in-place batched solve of fp64 right-hand sides

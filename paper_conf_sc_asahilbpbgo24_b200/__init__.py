@@ -12,7 +12,7 @@ from __future__ import annotations
 import ctypes
 
 from . import _lib
-from ._lib import (SB_F32, SB_F64, SB_FLAG_HOST_ONLY, SB_GREVILLE, SB_HERMITE, SB_PERIODIC, SplineBuilderError,
+from ._lib import (SB_F32, SB_F64, SB_FLAG_DEVICE_UPDATE, SB_FLAG_HOST_ONLY, SB_GREVILLE, SB_HERMITE, SB_PERIODIC, SplineBuilderError,
                    SplineBuilderInfo)
 
 PERIODIC, GREVILLE, HERMITE = SB_PERIODIC, SB_GREVILLE, SB_HERMITE
@@ -82,7 +82,7 @@ class SplineBuilder:
     GPU (inspection / CPU tests)."""
 
     def __init__(self, degree: int, n_points: int, bc: int = PERIODIC, knots=None, split=None,
-                 host_only: bool = False):
+                 host_only: bool = False, device_update: bool = False):
         lib = _lib.load()
         self._lib = lib
         kbuf = None
@@ -90,7 +90,7 @@ class SplineBuilder:
             self._knots = _knots_arg(knots, n_cells_of(degree, n_points, bc))
             kbuf = ctypes.c_void_p(self._knots.ctypes.data)
         lo, hi = (-1, -1) if split is None else split
-        flags = SB_FLAG_HOST_ONLY if host_only else 0
+        flags = (SB_FLAG_HOST_ONLY if host_only else 0) | (SB_FLAG_DEVICE_UPDATE if device_update else 0)
         h = lib.spline_builder_create_ex(int(degree), int(n_points), int(bc), kbuf, int(lo), int(hi), flags)
         if not h:
             raise SplineBuilderError(lib.spline_builder_last_status(), _lib.last_error())
@@ -128,6 +128,32 @@ class SplineBuilder:
         _lib.check(self._lib.spline_builder_update(self._h, kbuf))
         if knots is not None:
             self._knots = kn
+
+    def update_device_(self, knots=None, stream=None):
+        """New breakpoints factorised on the device (``spline_builder_update_device``;
+        handle created with ``device_update=True``): ``knots`` is a CUDA fp64
+        tensor of N+1 breakpoints (None: uniform).  Asynchronous on ``stream``;
+        :meth:`update_status` returns the outcome (the previous mesh is kept on
+        failure)."""
+        import torch
+        kp = None
+        if knots is not None:
+            if not (isinstance(knots, torch.Tensor) and knots.is_cuda and knots.dtype == torch.float64):
+                raise TypeError("knots must be a CUDA float64 tensor")
+            if knots.dim() != 1 or not knots.is_contiguous() or knots.numel() != self.info()["n_cells"] + 1:
+                raise ValueError(f"knots must be a contiguous 1-D tensor of N+1 = {self.info()['n_cells'] + 1} values")
+            self._dev_knots = knots  # kept alive until the kernel has read it
+            kp = ctypes.c_void_p(knots.data_ptr())
+        _lib.check(self._lib.spline_builder_update_device(self._h, kp, _stream_handle(stream)))
+        return self
+
+    def update_status(self) -> None:
+        """Wait for the last :meth:`update_device_`; raises SplineBuilderError if it
+        was rejected (the previous mesh stays in place)."""
+        try:
+            _lib.check(self._lib.spline_builder_update_status(self._h))
+        finally:
+            self._dev_knots = None
 
     # ------------------------------------------------------------- queries
     def info(self) -> dict:

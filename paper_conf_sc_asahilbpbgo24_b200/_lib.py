@@ -15,11 +15,12 @@ LIB_PATH = os.environ.get("SB_LIB_PATH") or os.path.join(HERE, "libsplinebuilder
 SB_PERIODIC, SB_GREVILLE, SB_HERMITE = 0, 1, 2
 SB_F64, SB_F32 = 0, 1
 SB_OK, SB_INVALID_ARG, SB_SINGULAR, SB_CUDA, SB_NOMEM, SB_UNSUPPORTED = range(6)
-SB_FLAG_HOST_ONLY = 1
+SB_FLAG_HOST_ONLY, SB_FLAG_DEVICE_UPDATE = 1, 2
 
 # every symbol include/spline_builder.h declares (checked by tests/test_abi.py)
 EXPORTS = [
-    "spline_builder_create", "spline_builder_create_ex", "spline_builder_update", "spline_builder_solve", "spline_builder_solve_f32",
+    "spline_builder_create", "spline_builder_create_ex", "spline_builder_update", "spline_builder_update_device",
+    "spline_builder_update_status", "spline_builder_solve", "spline_builder_solve_f32",
     "spline_builder_solve_strided", "spline_builder_solve_slabs", "spline_builder_solve_2d", "spline_builder_advect", "spline_builder_solve_host", "spline_builder_destroy",
     "spline_builder_get_info", "spline_builder_nbasis", "spline_builder_get_blocks",
     "spline_builder_solve_cpu_plan", "spline_builder_last_error", "spline_builder_last_status",
@@ -76,6 +77,10 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.spline_builder_solve_host.argtypes = [vp, dp, i32, i64, i64]
     lib.spline_builder_update.restype = i32
     lib.spline_builder_update.argtypes = [vp, dp]
+    lib.spline_builder_update_device.restype = i32
+    lib.spline_builder_update_device.argtypes = [vp, dp, vp]
+    lib.spline_builder_update_status.restype = i32
+    lib.spline_builder_update_status.argtypes = [vp]
     lib.spline_builder_destroy.restype = None
     lib.spline_builder_destroy.argtypes = [vp]
     lib.spline_builder_get_info.restype = i32

@@ -30,8 +30,9 @@ SOURCES = [
     ("warp_adv_f64.cu", "cu"),
     ("warp_adv_f32.cu", "cu"),
     ("serial.cu", "cu"),
+    ("refactor.cu", "cu"),
 ]
-HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh"]
+HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh", "refactor.hpp"]
 
 
 def _newer(target: str, deps: list[str]) -> bool:

@@ -16,6 +16,7 @@
 #include "../../include/spline_builder.h"
 #include "device.hpp"
 #include "host/plan.hpp"
+#include "refactor.hpp"
 
 namespace {
 
@@ -43,6 +44,16 @@ struct spline_builder {
     // CUDA graph before an update stay memory-safe (they keep the old mesh)
     std::vector<void *> retired;
     sb::DevPlan dp{};
+    // device-side refactorisation (SB_FLAG_DEVICE_UPDATE)
+    bool dev_update = false;
+    void *stage_blob = nullptr;   // staging copy of the blob (same layout)
+    void *rf_scratch = nullptr;   // scratch of the refactor kernel
+    int *rf_status = nullptr;     // device status word
+    int *rf_status_host = nullptr; // pinned copy of it
+    int *rf_rowdesc = nullptr;    // row descriptors (device)
+    cudaEvent_t rf_event = nullptr;
+    bool rf_pending = false;
+    double x0 = 0.0, xN = 1.0;    // periodic domain ends at create
     // staging for solve_host
     std::mutex host_mu;
     void *stage[3] = {nullptr, nullptr, nullptr};
@@ -106,7 +117,8 @@ int upload(spline_builder *h) {
         std::vector<int> slot(std::max(S, 1), 0), uniq;
         for (int s = 0; s < S; ++s) {
             int found = -1;
-            for (size_t u = 0; u < uniq.size() && found < 0; ++u)
+            // (device-updatable handles: one slot per segment, the factors change in place)
+            for (size_t u = 0; u < uniq.size() && found < 0 && !P.dev_update; ++u)
                 if (segdata[uniq[u]] == segdata[s]) found = (int)u;
             if (found < 0) { found = (int)uniq.size(); uniq.push_back(s); }
             slot[s] = found;
@@ -220,6 +232,42 @@ int upload(spline_builder *h) {
     return 0;
 }
 
+// device-update resources: a staging copy of the blob (initialised from the
+// live one, so the arrays the refactor kernel does not rewrite -- patterns,
+// slots -- are already in place), scratch, status word, row descriptors
+int init_device_update(spline_builder *h) {
+    const sb::Plan &P = h->plan;
+    auto bad = [&](cudaError_t e, const char *what) {
+        return fail(e == cudaErrorMemoryAllocation ? SB_NOMEM : SB_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+    };
+    cudaError_t e;
+    if (h->stage_blob) { cudaFree(h->stage_blob); h->stage_blob = nullptr; }
+    if ((e = cudaMalloc(&h->stage_blob, h->blob_bytes)) != cudaSuccess) return bad(e, "cudaMalloc(staging blob)");
+    if ((e = cudaMemcpy(h->stage_blob, h->blob, h->blob_bytes, cudaMemcpyDeviceToDevice)) != cudaSuccess)
+        return bad(e, "staging blob copy");
+    if (!h->rf_scratch &&
+        (e = cudaMalloc(&h->rf_scratch, sb::refactor_scratch_bytes(P.n, P.N, P.nQ, P.k, P.K))) != cudaSuccess)
+        return bad(e, "cudaMalloc(refactor scratch)");
+    if (!h->rf_status && (e = cudaMalloc(&h->rf_status, sizeof(int))) != cudaSuccess) return bad(e, "cudaMalloc(status)");
+    if (!h->rf_status_host && (e = cudaMallocHost(&h->rf_status_host, sizeof(int))) != cudaSuccess)
+        return bad(e, "cudaMallocHost(status)");
+    *h->rf_status_host = 0;
+    if (!h->rf_event && (e = cudaEventCreateWithFlags(&h->rf_event, cudaEventDisableTiming)) != cudaSuccess)
+        return bad(e, "cudaEventCreate");
+    std::vector<int> rd(3 * P.n);
+    for (int i = 0; i < P.n; ++i) {
+        rd[3 * i] = P.rowdesc[i].kind; rd[3 * i + 1] = P.rowdesc[i].idx; rd[3 * i + 2] = P.rowdesc[i].deriv;
+    }
+    if (h->rf_rowdesc) { cudaFree(h->rf_rowdesc); h->rf_rowdesc = nullptr; }
+    if ((e = cudaMalloc(&h->rf_rowdesc, rd.size() * sizeof(int))) != cudaSuccess) return bad(e, "cudaMalloc(rowdesc)");
+    if ((e = cudaMemcpy(h->rf_rowdesc, rd.data(), rd.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess)
+        return bad(e, "rowdesc upload");
+    if ((e = cudaStreamSynchronize(0)) != cudaSuccess) return bad(e, "device-update setup");
+    h->x0 = P.xb.empty() ? 0.0 : P.xb[0];
+    h->xN = P.xb.empty() ? 1.0 : P.xb[P.N];
+    return SB_OK;
+}
+
 int do_solve(spline_builder *h, void *rhs, int dtype, int64_t batch, int64_t bstride, int64_t pstride,
              cudaStream_t stream, const double *shift = nullptr, int64_t nslab = 1, int64_t slab_stride = 0) {
     if (!h) return fail(SB_INVALID_ARG, "null handle");
@@ -267,7 +315,8 @@ spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, cons
     spline_builder *h = new (std::nothrow) spline_builder();
     if (!h) { fail(SB_NOMEM, "out of host memory"); return nullptr; }
     try {
-        sb::Status st = sb::build_plan(h->plan, degree, n_points, bc, knots, split_lo, split_hi);
+        const int pflags = (flags & SB_FLAG_DEVICE_UPDATE) ? sb::PLAN_DEVICE_UPDATE : 0;
+        sb::Status st = sb::build_plan(h->plan, degree, n_points, bc, knots, split_lo, split_hi, pflags);
         if (st.code) { fail(st.code, st.msg); delete h; return nullptr; }
     } catch (const std::bad_alloc &) {
         fail(SB_NOMEM, "out of host memory in create"); delete h; return nullptr;
@@ -275,11 +324,13 @@ spline_builder_t spline_builder_create_ex(int degree, int n_points, int bc, cons
         fail(SB_INVALID_ARG, "unexpected failure in create"); delete h; return nullptr;
     }
     h->host_only = (flags & SB_FLAG_HOST_ONLY) != 0;
+    h->dev_update = (flags & SB_FLAG_DEVICE_UPDATE) != 0;
     h->c_degree = degree; h->c_npoints = n_points; h->c_bc = bc; h->c_split_lo = split_lo; h->c_split_hi = split_hi;
     if (!h->host_only) {
         if (cudaGetDevice(&h->device) != cudaSuccess) { fail(SB_CUDA, "no CUDA device"); delete h; return nullptr; }
         cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device);
         if (upload(h)) { spline_builder_destroy(h); return nullptr; }
+        if (h->dev_update && init_device_update(h)) { spline_builder_destroy(h); return nullptr; }
     }
     return h;
 }
@@ -288,7 +339,8 @@ int spline_builder_update(spline_builder_t h, const double *knots) {
     if (!h) return fail(SB_INVALID_ARG, "null handle");
     sb::Plan fresh;
     try {
-        sb::Status st = sb::build_plan(fresh, h->c_degree, h->c_npoints, h->c_bc, knots, h->c_split_lo, h->c_split_hi);
+        sb::Status st = sb::build_plan(fresh, h->c_degree, h->c_npoints, h->c_bc, knots, h->c_split_lo, h->c_split_hi,
+                                       h->dev_update ? sb::PLAN_DEVICE_UPDATE : 0);
         if (st.code) return fail(st.code, st.msg);
     } catch (const std::bad_alloc &) {
         return fail(SB_NOMEM, "out of host memory in update");
@@ -315,8 +367,72 @@ int spline_builder_update(spline_builder_t h, const double *knots) {
         return fail(rc, msg);
     }
     if (old_blob) h->retired.push_back(old_blob);  // freed at destroy (graphs may still reference it)
+    int rc2 = SB_OK;
+    if (h->dev_update) rc2 = init_device_update(h);  // new layout: fresh staging copy
     if (cur != h->device) cudaSetDevice(cur);
+    return rc2;
+}
+
+int spline_builder_update_device(spline_builder_t h, const double *knots, void *stream) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (h->host_only) return fail(SB_UNSUPPORTED, "handle was created with SB_FLAG_HOST_ONLY");
+    if (!h->dev_update) return fail(SB_UNSUPPORTED, "handle was not created with SB_FLAG_DEVICE_UPDATE");
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != h->device) cudaSetDevice(h->device);
+    sb::RefactorArgs a{};
+    a.P = h->dp;
+    a.p = h->plan.p;
+    a.x0 = h->x0; a.xN = h->xN;
+    a.knots = knots;
+    a.rowdesc = h->rf_rowdesc;
+    a.lam_ptr = h->dp.lam_ptr; a.lam_c = h->dp.lam_c; a.gam_r = h->dp.gam_r; a.gam_c = h->dp.gam_c;
+    a.drow = h->dp.drow;
+    a.scr = static_cast<double *>(h->rf_scratch);
+    a.stage = static_cast<unsigned char *>(h->stage_blob);
+    a.live = static_cast<unsigned char *>(h->blob);
+    a.blob_bytes = h->blob_bytes / 16 * 16;
+    a.status = h->rf_status;
+    char err[256] = {0};
+    const cudaStream_t st = (cudaStream_t)stream;
+    int rc = sb::launch_refactor(a, st, err, sizeof(err));
+    cudaError_t e = cudaSuccess;
+    if (!rc) e = cudaMemcpyAsync(h->rf_status_host, h->rf_status, sizeof(int), cudaMemcpyDeviceToHost, st);
+    if (!rc && e == cudaSuccess) e = cudaEventRecord(h->rf_event, st);
+    if (cur != h->device) cudaSetDevice(cur);
+    if (rc) return fail(rc, err);
+    if (e != cudaSuccess) return fail(SB_CUDA, std::string("update_device: ") + cudaGetErrorString(e));
+    h->rf_pending = true;
     return SB_OK;
+}
+
+int spline_builder_update_status(spline_builder_t h) {
+    if (!h) return fail(SB_INVALID_ARG, "null handle");
+    if (!h->dev_update || !h->rf_pending) return SB_OK;
+    const cudaError_t e = cudaEventSynchronize(h->rf_event);
+    if (e != cudaSuccess) return fail(SB_CUDA, std::string("update_status: ") + cudaGetErrorString(e));
+    h->rf_pending = false;
+    switch (*h->rf_status_host) {
+        case sb::SB_RF_OK: return SB_OK;
+        case sb::SB_RF_BADKNOTS: return fail(SB_INVALID_ARG, "device update: breakpoints must be strictly increasing");
+        case sb::SB_RF_DOMAIN: return fail(SB_INVALID_ARG, "device update: a periodic mesh must keep its end points");
+        case sb::SB_RF_SINGULAR: return fail(SB_SINGULAR, "device update: Q or delta' could not be factored");
+        case sb::SB_RF_CARRY:
+            return fail(SB_UNSUPPORTED, "device update: the new mesh needs deeper segment carries than frozen at create");
+        case sb::SB_RF_LAMBDA:
+            return fail(SB_UNSUPPORTED, "device update: Lambda has entries above 1e-14 outside the pattern frozen at "
+                                        "create (use spline_builder_update)");
+        case sb::SB_RF_GAMMA:
+            return fail(SB_UNSUPPORTED, "device update: gamma leaves the pattern frozen at create (use spline_builder_update)");
+        case sb::SB_RF_BUCKETS:
+            return fail(SB_UNSUPPORTED, "device update: the new cells are too small for the advection bucket table "
+                                        "frozen at create (use spline_builder_update)");
+        case sb::SB_RF_SCALED:
+            return fail(SB_UNSUPPORTED, "device update: a derivative row fell into Q (use spline_builder_update)");
+        default:
+            return fail(SB_UNSUPPORTED, "device update: the new collocation matrix leaves the Q band frozen at create "
+                                        "(use spline_builder_update)");
+    }
 }
 
 spline_builder_t spline_builder_create(int degree, int n_points, int bc, const double *knots) {
@@ -469,6 +585,12 @@ void spline_builder_destroy(spline_builder_t h) {
         if (h->device >= 0 && cur != h->device) cudaSetDevice(h->device);
         if (h->blob) cudaFree(h->blob);
         for (void *b : h->retired) cudaFree(b);
+        if (h->stage_blob) cudaFree(h->stage_blob);
+        if (h->rf_scratch) cudaFree(h->rf_scratch);
+        if (h->rf_status) cudaFree(h->rf_status);
+        if (h->rf_rowdesc) cudaFree(h->rf_rowdesc);
+        if (h->rf_status_host) cudaFreeHost(h->rf_status_host);
+        if (h->rf_event) cudaEventDestroy(h->rf_event);
         for (int i = 0; i < 3; ++i) {
             if (h->stage[i]) cudaFree(h->stage[i]);
             if (h->streams[i]) cudaStreamDestroy(h->streams[i]);

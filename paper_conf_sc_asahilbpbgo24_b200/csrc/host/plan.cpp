@@ -150,7 +150,7 @@ SplitResult try_split(Plan &P, int slo, int shi) {
         const SparseRow &row = P.A[slo + i];
         for (size_t e = 0; e < row.col.size(); ++e) {
             int c = row.col[e];
-            if (c < slo || c >= n - shi || row.val[e] == 0.0) continue;
+            if (c < slo || c >= n - shi || (row.val[e] == 0.0 && !P.dev_update)) continue;
             int o = (c - slo) - i;
             kl = std::max(kl, -o);
             ku = std::max(ku, o);
@@ -326,9 +326,23 @@ SplitResult try_split(Plan &P, int slo, int shi) {
                 P.lam_r.push_back(r); P.lam_c.push_back(i); P.lam_v.push_back(lam[(size_t)r * nQ + i]);
             }
     P.gam_r.clear(); P.gam_c.clear(); P.gam_v.clear();
+    // PLAN_DEVICE_UPDATE: the gamma pattern is frozen at create, so it covers every
+    // delta column of the rows within CORNER_MARGIN of a structural nonzero (a new
+    // mesh may move a collocation point into a neighbouring span)
+    std::vector<char> grow(nQ, 0);
     for (int i = 0; i < nQ; ++i)
         for (int c = 0; c < k; ++c)
-            if (gam[(size_t)i * k + c] != 0.0) {
+            if (gam[(size_t)i * k + c] != 0.0) grow[i] = 1;
+    if (P.dev_update) {
+        std::vector<char> g2(nQ, 0);
+        for (int i = 0; i < nQ; ++i)
+            if (grow[i])
+                for (int j = std::max(0, i - CORNER_MARGIN); j <= std::min(nQ - 1, i + CORNER_MARGIN); ++j) g2[j] = 1;
+        grow.swap(g2);
+    }
+    for (int i = 0; i < nQ; ++i)
+        for (int c = 0; c < k; ++c)
+            if (gam[(size_t)i * k + c] != 0.0 || (P.dev_update && grow[i])) {
                 P.gam_r.push_back(i); P.gam_c.push_back(c); P.gam_v.push_back(gam[(size_t)i * k + c]);
             }
     P.beta_r.clear(); P.beta_c.clear(); P.beta_v.clear();
@@ -338,11 +352,22 @@ SplitResult try_split(Plan &P, int slo, int shi) {
             if (std::fabs(b) > CORNER_DROP) { P.beta_r.push_back(i); P.beta_c.push_back(c); P.beta_v.push_back(b); }
         }
     P.Lam_ptr.assign(k + 1, 0); P.Lam_c.clear(); P.Lam_v.clear();
+    // PLAN_DEVICE_UPDATE: one frozen column set for every row of Lambda (the union
+    // of the rows' columns above the threshold, dilated by CORNER_MARGIN columns):
+    // a row whose entries at one end fall just under 1e-14 on this mesh may have
+    // them above it on the next
+    std::vector<char> uni(nQ, 0);
+    if (P.dev_update)
+        for (int d = 0; d < k; ++d)
+            for (int i = 0; i < nQ; ++i)
+                if (std::fabs(Lam[(size_t)d * nQ + i]) > CORNER_DROP)
+                    for (int j = std::max(0, i - CORNER_MARGIN); j <= std::min(nQ - 1, i + CORNER_MARGIN); ++j) uni[j] = 1;
     for (int d = 0; d < k; ++d) {
-        for (int i = 0; i < nQ; ++i) {
-            double l = Lam[(size_t)d * nQ + i];
-            if (std::fabs(l) > CORNER_DROP) { P.Lam_c.push_back(i); P.Lam_v.push_back(l); }
-        }
+        for (int i = 0; i < nQ; ++i)
+            if (P.dev_update ? uni[i] != 0 : std::fabs(Lam[(size_t)d * nQ + i]) > CORNER_DROP) {
+                P.Lam_c.push_back(i);
+                P.Lam_v.push_back(Lam[(size_t)d * nQ + i]);
+            }
         P.Lam_ptr[d + 1] = (int)P.Lam_c.size();
     }
     return R;
@@ -409,7 +434,7 @@ void build_segplan(const Plan &P, SegPlan &G, int L) {
             prod *= nrm(G.G, t);
             if (prod <= eps) break;
         }
-        G.carry_f = std::max(G.carry_f, T);
+        G.carry_f = std::max(G.carry_f, T + (P.dev_update && T < s ? 1 : 0));  // device update: one deeper
     }
     G.carry_b = 0;
     for (int s = 0; s + 1 < S; ++s) {
@@ -422,7 +447,7 @@ void build_segplan(const Plan &P, SegPlan &G, int L) {
             prod *= nrm(G.H, t);
             if (prod <= eps) break;
         }
-        G.carry_b = std::max(G.carry_b, T);
+        G.carry_b = std::max(G.carry_b, T + (P.dev_update && s + T < S - 1 ? 1 : 0));
     }
 }
 
@@ -569,7 +594,7 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
             xmax = std::max(xmax, std::fabs(P.xb[c]));
         }
         for (int i = 0; i < n; ++i) dev = std::max(dev, std::fabs((P.xi[i] - P.xi[0]) - i * hu));
-        P.adv_uniform = dev <= 2.3e-16 * xmax;
+        P.adv_uniform = dev <= 2.3e-16 * xmax && !P.dev_update;  // device update: generic geometry
         P.adv_invh = 1.0 / hu;
         P.adv_q0 = (P.xi[0] - P.xb[0]) / hu;
         // bucket table: buckets no wider than the smallest cell (up to 8N of them);
@@ -579,7 +604,10 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         {
             double hmin = Lp;
             for (int c = 0; c < N; ++c) hmin = std::min(hmin, P.xb[c + 1] - P.xb[c]);
-            const int MT = std::max(1, (int)std::min<double>(8.0 * N, std::ceil(Lp / hmin * (1.0 + 1e-12))));
+            // (device update: twice as many buckets, so a new mesh whose smallest cell
+            // is down to half of this one keeps the frozen step count)
+            const double fine = P.dev_update ? 2.0 : 1.0;
+            const int MT = std::max(1, (int)std::min<double>(8.0 * N, std::ceil(fine * Lp / hmin * (1.0 + 1e-12))));
             const double w = Lp / MT, margin = 1e-9 * w;
             auto cell_of = [&](double x) {  // t_c <= x < t_{c+1}, clamped to [0, N)
                 int lo = 0, hi = N - 1;
@@ -598,6 +626,9 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
                 P.adv_tbl[b] = lo;
                 P.adv_steps = std::max(P.adv_steps, hi - lo);
             }
+            // device update: two more locate steps, so cells down to a third of the
+            // bucket width (jitter +-0.3h on a 2x finer table) keep the frozen table
+            if (P.dev_update) P.adv_steps += 2;
         }
         // reciprocal knot differences 1/(t_{m+w} - t_m), m in [-p, N+p), w = 1..p:
         // the denominators of de Boor's recursion depend on the knots only, so the
@@ -616,8 +647,19 @@ Status build_plan(Plan &P, int degree, int n_points, int bc, const double *knots
         else bsplvd(S, rows[i].span, rows[i].u, rows[i].deriv, vals);
         std::map<int, double> acc;
         for (int r = 0; r <= p; ++r) acc[S.basis_of(rows[i].span - p + r)] += vals[r] * P.rowscale[i];
+        if (P.dev_update) {
+            // structure frozen for later meshes: a Greville point that sits ON a knot
+            // (uniform odd-degree meshes put every one there) moves into the
+            // neighbouring span under any perturbation, so the basis function on that
+            // side is a structural entry (value 0 here) of the band and the split
+            const double w = S.width(rows[i].span), u = rows[i].u;
+            if (P.rowdesc[i].kind == ROW_GREVILLE && u <= 1e-12 * w) {  // (break / end rows stay on their knot)
+                const long q = rows[i].span - p - 1;
+                if (bc == PERIODIC || q >= 0) acc[S.basis_of(q)] += 0.0;
+            }
+        }
         for (auto &kv : acc)
-            if (kv.second != 0.0) { P.A[i].col.push_back(kv.first); P.A[i].val.push_back(kv.second); }
+            if (kv.second != 0.0 || P.dev_update) { P.A[i].col.push_back(kv.first); P.A[i].val.push_back(kv.second); }
         if (P.A[i].col.empty()) return {2, "empty collocation row"};
     }
     // candidate splits

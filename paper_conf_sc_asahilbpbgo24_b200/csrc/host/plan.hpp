@@ -37,7 +37,7 @@ enum PlanFlags {
                             // CORNER_MARGIN, carry walks one segment deeper, no slot sharing, generic
                             // (non-uniform) advection geometry with a 2x finer bucket table
 };
-constexpr int CORNER_MARGIN = 16;  // Lambda columns / gamma rows kept around the create-time pattern
+constexpr int CORNER_MARGIN = 24;  // Lambda columns / gamma rows kept around the create-time pattern
 
 struct SparseRow {
     std::vector<int> col;

@@ -586,3 +586,145 @@ def test_two_host_threads_two_streams_one_handle(torch_cuda):
     for i in range(2):
         assert kernels[i].startswith("tile<f64") and "TMA" in kernels[i], kernels[i]
         assert rel_coef_error(ts[i].cpu().numpy(), o.solve(bs[i])) <= TOL64
+
+
+# ------------------------------------------------------------ device-side refactorisation
+DEV_UPDATE_CASES = [
+    # (degree, n_points, bc, create mesh, new meshes)
+    (3, 1000, PERIODIC, "sin", ["jitter", "sin2", "uniform_array"]),
+    (3, 1000, PERIODIC, "uniform", ["jitter"]),
+    (4, 600, PERIODIC, "jitter", ["sin"]),
+    (5, 1000, GREVILLE, "sin", ["jitter", "sin2"]),
+    (5, 996, HERMITE, "sin", ["jitter", "sin2"]),
+    (3, 200, GREVILLE | (HERMITE << 4), "jitter", ["sin"]),
+]
+
+
+def _mesh(N, kind):
+    if kind == "sin2":  # the sin map with a smaller amplitude: another smooth non-uniform mesh
+        u = np.arange(N + 1, dtype=np.float64) / N
+        x = u + 0.3 * np.sin(2.0 * np.pi * u) / (2.0 * np.pi)
+        x[0], x[-1] = 0.0, 1.0
+        return x
+    x = inputs.breakpoints(N, kind)
+    return x if x is not None else inputs.breakpoints(N, "uniform_array")
+
+
+@pytest.mark.parametrize("case", DEV_UPDATE_CASES, ids=lambda c: f"p{c[0]}-n{c[1]}-bc{c[2]}-{c[3]}")
+def test_update_device_new_meshes_parity(torch_cuda, case):
+    """spline_builder_update_device: the factorisation of a new
+    mesh is computed by a kernel on the device; the batched solve (tile kernel,
+    batch-contiguous, and warp kernel, point layout) then matches the oracle
+    built on the new breakpoints, element by element at 1e-12, plus the
+    interpolation residual."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder
+    p, npts, bc, m0, news = case
+    N = inputs.n_cells(p, npts, bc)
+    sb = SplineBuilder(p, npts, bc, _mesh(N, m0), device_update=True)
+    b = inputs.rhs(sb.n, 777, seed=31, degree=p, bc=bc)
+    for kind in news:
+        x = _mesh(N, kind)
+        sb.update_device_(torch.from_numpy(x).cuda())
+        sb.update_status()
+        o = Oracle(p, npts, bc, x)
+        ref = o.solve(b)
+        got = gpu_solve(torch, sb, b)
+        assert rel_coef_error(got, ref) <= TOL64, (kind, rel_coef_error(got, ref))
+        assert o.residual(got, b) <= TOL64
+        t = torch.from_numpy(np.ascontiguousarray(b.T)).cuda()
+        sb.solve_(t)
+        torch.cuda.synchronize()
+        assert rel_coef_error(np.ascontiguousarray(t.cpu().numpy().T), ref) <= TOL64, kind
+
+
+def test_update_device_advection_and_graph_replay(torch_cuda):
+    """After a device update the advection step (non-uniform evaluation data
+    rebuilt on the device) matches the oracle on the new mesh, and a solve
+    captured in a CUDA graph BEFORE the update replays with the new mesh (the
+    launch arguments point at constants updated in place)."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder
+    N = 1024
+    x0, x1 = _mesh(N, "sin"), _mesh(N, "jitter")
+    sb = SplineBuilder(3, N, PERIODIC, x0, device_update=True)
+    b = inputs.rhs(N, 4096, seed=41)
+    t = torch.from_numpy(b).cuda()
+    pristine = t.clone()
+    g = torch.cuda.CUDAGraph()
+    sb.solve_(t)  # warm-up outside the capture
+    with torch.cuda.graph(g):
+        sb.solve_(t)
+    sb.update_device_(torch.from_numpy(x1).cuda())
+    sb.update_status()
+    t.copy_(pristine)
+    g.replay()
+    torch.cuda.synchronize()
+    o1 = Oracle(3, N, PERIODIC, x1)
+    assert rel_coef_error(t.cpu().numpy(), o1.solve(b)) <= TOL64
+    B = 300
+    f = inputs.rhs(N, B, seed=43)
+    shift = np.linspace(-2.0, 2.0, B) / N
+    tf = torch.from_numpy(np.ascontiguousarray(f.T)).cuda()
+    sb.advect_(tf, torch.from_numpy(shift).cuda())
+    torch.cuda.synchronize()
+    assert rel_coef_error(np.ascontiguousarray(tf.cpu().numpy().T), o1.advect(f, shift)) <= TOL64
+
+
+def test_update_device_rejections_keep_previous_mesh(torch_cuda):
+    """The status path of the device update: knots that are not increasing
+    (SB_INVALID_ARG), a periodic mesh that moves its end points
+    (SB_INVALID_ARG), and a mesh whose matrix leaves the structure frozen at
+    create (SB_UNSUPPORTED: a Lambda entry above 1e-14 outside the pattern) are
+    rejected on the device; the previous mesh stays live and solves still
+    match its oracle."""
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, SplineBuilderError
+    N = 500
+    x0 = _mesh(N, "sin")
+    sb = SplineBuilder(3, N, PERIODIC, x0, device_update=True)
+    o0 = Oracle(3, N, PERIODIC, x0)
+    b = inputs.rhs(N, 64, seed=51)
+    bad = x0.copy()
+    bad[10], bad[11] = bad[11], bad[10]
+    moved = x0 * 2.0
+    # cells shrinking geometrically towards x = 0.5: far slower decay of Lambda
+    # than the create-time mesh, so entries above 1e-14 appear outside the pattern
+    u = np.arange(N + 1) / N
+    steep = 0.5 + 0.5 * np.sign(u - 0.5) * np.abs(2 * u - 1) ** 6
+    expected = [(bad, 1), (moved, 1), (steep, 5)]
+    for x, status in expected:
+        sb.update_device_(torch.from_numpy(x).cuda())
+        with pytest.raises(SplineBuilderError) as ei:
+            sb.update_status()
+        assert ei.value.status == status, (status, str(ei.value))
+        assert rel_coef_error(gpu_solve(torch, sb, b), o0.solve(b)) <= TOL64
+
+
+def test_update_device_faster_than_host_replan(torch_cuda):
+    """The device refactorisation of a C3 Greville mesh (n = 1000, p = 5) takes
+    less time than the host re-plan + upload of spline_builder_update (the
+    point of the device path: meshes that change every step)."""
+    import time
+    torch = torch_cuda
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder
+    N = inputs.n_cells(5, 1000, GREVILLE)
+    xs = [_mesh(N, k) for k in ("sin", "sin2")]
+    sb = SplineBuilder(5, 1000, GREVILLE, xs[0], device_update=True)
+    dx = [torch.from_numpy(x).cuda() for x in xs]
+    for i in range(3):
+        sb.update_device_(dx[i % 2])
+        sb.update_status()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    reps = 20
+    for i in range(reps):
+        sb.update_device_(dx[i % 2])
+    sb.update_status()
+    t_dev = (time.perf_counter() - t0) / reps
+    t0 = time.perf_counter()
+    for i in range(5):
+        sb.update(xs[i % 2])
+    t_host = (time.perf_counter() - t0) / 5
+    print(f"device update {t_dev * 1e3:.3f} ms, host re-plan {t_host * 1e3:.3f} ms")
+    assert t_dev < t_host
