@@ -154,6 +154,17 @@ __device__ void band_lu_window(double *W, int nQ, double qmax, int *st, double &
         for (int c = 0; c <= K; ++c) A[r][c] = (r < nQ && c < nQ) ? W[r * BW + (c - r + K)] : 0.0;
     lmax = umax = 0.0;
     for (int j = 0; j < nQ; ++j) {
+        // the entries entering the window after this step (never written by it): loaded
+        // first, so they are in flight during the step's dependent reciprocal / FMAs
+        const int nr = j + K + 1;
+        double nrow[K + 1], ncol[K];
+#pragma unroll
+        for (int c = 0; c <= K; ++c) nrow[c] = nr < nQ ? W[(size_t)nr * BW + c] : 0.0;
+#pragma unroll
+        for (int r = 0; r < K; ++r) {
+            const int row = j + 1 + r;
+            ncol[r] = (row < nQ && nr < nQ) ? W[(size_t)row * BW + K + (K - r)] : 0.0;
+        }
         const double pv = A[0][0];
         if (!(fabs(pv) > 1e-13 * qmax)) { fail(st, SB_RF_SINGULAR); return; }
         const double rp = 1.0 / pv;
@@ -177,14 +188,11 @@ __device__ void band_lu_window(double *W, int nQ, double qmax, int *st, double &
         for (int r = 0; r < K; ++r)
 #pragma unroll
             for (int c = 0; c < K; ++c) A[r][c] = A[r + 1][c + 1];
-        const int nr = j + K + 1;  // new last row, columns j+1 .. j+K+1 (offsets -K .. 0)
+        // new last row j+K+1 (columns j+1 .. j+K+1) and new last column j+K+1 (rows j+1 .. j+K)
 #pragma unroll
-        for (int c = 0; c <= K; ++c) A[K][c] = nr < nQ ? W[(size_t)nr * BW + c] : 0.0;
+        for (int c = 0; c <= K; ++c) A[K][c] = nrow[c];
 #pragma unroll
-        for (int r = 0; r < K; ++r) {  // new last column j+K+1 of rows j+1 .. j+K (offset K - r)
-            const int row = j + 1 + r;
-            A[r][K] = (row < nQ && nr < nQ) ? W[(size_t)row * BW + K + (K - r)] : 0.0;
-        }
+        for (int r = 0; r < K; ++r) A[r][K] = ncol[r];
     }
 }
 
@@ -317,24 +325,25 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
         const int c = tid;
         double win[K];
         {  // Lambda(c, :): Q^T w = lambda(c, :)^T with Q = L D (I + U'), in place in lam
-            double *w = Lam + (size_t)c * nQ;
+            double *__restrict__ w = Lam + (size_t)c * nQ;
+            const double *__restrict__ Qr = Qb;  // the factors: loads may run ahead of the stores to w
 #pragma unroll
             for (int m = 0; m < K; ++m) win[m] = 0.0;  // win[m] = w_{j-1-m}
             for (int j = 0; j < nQ; ++j) {
                 double acc = w[j];
 #pragma unroll
-                for (int m = K; m >= 1; --m) acc = j - m >= 0 ? fma(-UB(j - m, m), win[m - 1], acc) : acc;
+                for (int m = K; m >= 1; --m) acc = j - m >= 0 ? fma(-Qr[(size_t)(j - m) * BW + K + m], win[m - 1], acc) : acc;
 #pragma unroll
                 for (int m = K - 1; m > 0; --m) win[m] = win[m - 1];
                 win[0] = acc;
-                w[j] = acc * DINV(j);
+                w[j] = acc * Qr[(size_t)j * BW + K];
             }
 #pragma unroll
             for (int m = 0; m < K; ++m) win[m] = 0.0;  // win[m] = w_{j+1+m}
             for (int j = nQ - 1; j >= 0; --j) {
                 double acc = w[j];
 #pragma unroll
-                for (int m = K; m >= 1; --m) acc = j + m < nQ ? fma(-LB(j + m, m), win[m - 1], acc) : acc;
+                for (int m = K; m >= 1; --m) acc = j + m < nQ ? fma(-Qr[(size_t)(j + m) * BW + K - m], win[m - 1], acc) : acc;
 #pragma unroll
                 for (int m = K - 1; m > 0; --m) win[m] = win[m - 1];
                 win[0] = acc;
@@ -384,17 +393,20 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
             double *F8 = S8(G.F[0]);
             float *F4 = S4(G.F[1]);
             const size_t BS = (size_t)BW * LP;
-            for (size_t e = tid; e < (size_t)G.nslots * BS; e += nth) {
-                const int s = (int)(e / BS), b = (int)((e % BS) / LP), i = (int)(e % LP);
-                const int row = s * L + i;
-                double v = b == 2 * K ? 1.0 : 0.0;
-                if (i < L && row < nQ) {
-                    if (b < K) v = LB(row, b + 1);
-                    else if (b < 2 * K) v = UB(row, b - K + 1);
-                    else v = DINV(row);
+            for (int sb = tid; sb < G.nslots * BW; sb += nth) {  // one factor row (slot s, band b) per thread
+                const int s = sb / BW, b = sb - s * BW;
+                const size_t e0 = (size_t)s * BS + (size_t)b * LP;
+                for (int i = 0; i < LP; ++i) {
+                    const int row = s * L + i;
+                    double v = b == 2 * K ? 1.0 : 0.0;
+                    if (i < L && row < nQ) {
+                        if (b < K) v = LB(row, b + 1);
+                        else if (b < 2 * K) v = UB(row, b - K + 1);
+                        else v = DINV(row);
+                    }
+                    F8[e0 + i] = v;
+                    F4[e0 + i] = (float)v;
                 }
-                F8[e] = v;
-                F4[e] = (float)v;
             }
             double *G8 = S8(G.G[0]), *H8 = S8(G.H[0]);
             float *G4 = S4(G.G[1]), *H4 = S4(G.H[1]);
@@ -502,18 +514,16 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
         }
         // corner data: Lambda CSR values on the frozen pattern (+ pattern check),
         // its dense window, gamma COO values (+ check), delta' LU, row scales
-        if (tid < k) {
-            const int d = tid;
+        {   // values on the pattern, then: no entry above the threshold off the pattern
+            // (the pattern's entries of Lambda are zeroed after being read)
             double *LV8 = S8(P.lam_v[0]);
             float *LV4 = S4(P.lam_v[1]);
-            int e = a.lam_ptr[d];
-            const int e1 = a.lam_ptr[d + 1];
-            for (int i = 0; i < nQ; ++i) {
-                const double v = Lam[(size_t)d * nQ + i];
-                const bool in = e < e1 && a.lam_c[e] == i;
-                if (in) { LV8[e] = v; LV4[e] = (float)v; ++e; }
-                else if (fabs(v) > CORNER_DROP_D) fail(st, SB_RF_LAMBDA);
-            }
+            for (int d = 0; d < k; ++d)
+                for (int e = a.lam_ptr[d] + tid; e < a.lam_ptr[d + 1]; e += nth) {
+                    const double v = Lam[(size_t)d * nQ + a.lam_c[e]];
+                    LV8[e] = v;
+                    LV4[e] = (float)v;
+                }
         }
         {
             const int lh = P.lw_head, lw = P.lw_head + P.lw_tail;
@@ -521,15 +531,20 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
             float *W4 = S4(P.lw_v[1]);
             for (int e = tid; e < lw * k; e += nth) { W8[e] = 0.0; W4[e] = 0.f; }
             __syncthreads();
-            if (tid < k) {
-                const int d = tid;
-                for (int e = a.lam_ptr[d]; e < a.lam_ptr[d + 1]; ++e) {
+            for (int d = 0; d < k; ++d) {
+                for (int e = a.lam_ptr[d] + tid; e < a.lam_ptr[d + 1]; e += nth) {
                     const int c = a.lam_c[e];
                     const int j = c < lh ? c : lh + (c - (nQ - P.lw_tail));
                     const double v = Lam[(size_t)d * nQ + c];
                     if (j >= 0 && j < lw) { W8[(size_t)j * k + d] = v; W4[(size_t)j * k + d] = (float)v; }
                 }
             }
+            __syncthreads();
+            for (int d = 0; d < k; ++d)
+                for (int e = a.lam_ptr[d] + tid; e < a.lam_ptr[d + 1]; e += nth) Lam[(size_t)d * nQ + a.lam_c[e]] = 0.0;
+            __syncthreads();
+            for (int i = tid; i < k * nQ; i += nth)
+                if (fabs(Lam[i]) > CORNER_DROP_D) fail(st, SB_RF_LAMBDA);
         }
         {
             double *GV8 = S8(P.gam_v[0]);
