@@ -445,6 +445,80 @@ def run_reference(args, wl):
     print(json.dumps(line), flush=True)
 
 
+EXTRA_DEFAULT = "C1,C3G,C3H,C4,C4F32,C4M,ADV,ADVNU,C5,C6"
+
+
+def quick_measure(name, steps=20, warmup=3):
+    """One device-timed measurement of another workload on this GPU (same
+    protocol as the headline: CUDA graph of `steps` launches, input restored
+    and L2 flushed before the timed chunk, CUDA events on the launching
+    stream), for the `extra_workloads` record of the default run: so the
+    round-end bench line carries every BASELINE config (C1-C5) and the NEXT
+    rows, not only C2.  Returns a small dict (no e2e / CPU baseline)."""
+    import torch
+    from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, last_kernel, solve_2d_
+    stream = torch.cuda.current_stream()
+    peak, _ = load_peaks()
+    if name in TWOD:
+        spec1, spec2, G, dt, desc = TWOD[name]
+        sbs = [SplineBuilder(d, p_, b, inputs.breakpoints(inputs.n_cells(d, p_, b), m)) for d, p_, b, m in (spec1, spec2)]
+        n1, n2 = sbs[0].n, sbs[1].n
+        host = np.ascontiguousarray(inputs.rhs(n1, G * n2, seed=1234).T.reshape(G, n2, n1).astype(
+            np.float32 if dt == "f32" else np.float64))
+        pristine = torch.from_numpy(host).cuda()
+        x = pristine.clone()
+        step = lambda: solve_2d_(sbs[0], sbs[1], x)  # noqa: E731
+        restore = lambda: x.copy_(pristine)  # noqa: E731
+        units, unit, esz, n_el = n1 * n2 * G, "points/s", (4 if dt == "f32" else 8), n1 * n2 * G
+        kern = "warp pass + tile slab pass"
+    else:
+        deg, npts, bc, mesh, B, dt, layout, desc = WORKLOADS[name]
+        n = inputs.nbasis(deg, npts, bc)
+        sb = SplineBuilder(deg, npts, bc, inputs.breakpoints(inputs.n_cells(deg, npts, bc), mesh))
+        tdt = torch.float32 if dt == "f32" else torch.float64
+        if n * B > DEVICE_INPUT_ELEMS and layout == "batch":
+            x = inputs.rhs_device(n, B, seed=1234, dtype=tdt)
+            restore = lambda: inputs.rhs_device(n, B, seed=1234, dtype=tdt, out=x)  # noqa: E731
+        else:
+            pristine = torch.from_numpy(make_rhs(deg, n, bc, B, 0, layout, dt)).cuda()
+            x = pristine.clone()
+            restore = lambda: x.copy_(pristine)  # noqa: E731
+        if name in ADVECT:
+            sh = torch.from_numpy(adv_shift(inputs.n_cells(deg, npts, bc), B)).cuda()
+            step = lambda: sb.advect_(x, sh)  # noqa: E731
+        elif layout == "slabs":
+            step = lambda: sb.solve_slabs_(x, SLAB_W, SLAB_W, B // SLAB_W, n * SLAB_W)  # noqa: E731
+        else:
+            step = lambda: sb.solve_(x)  # noqa: E731
+        esz = 4 if dt == "f32" else 8
+        units, unit, n_el = B, "RHS/s", n * B
+        if name in ADVECT:
+            units, unit = B * n / 1e9, "GLUPS"
+    for _ in range(warmup):
+        step()
+    kern = last_kernel() if name not in TWOD else kern
+    runner = ChunkRunner(step, True)
+    runner(steps)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    restore()
+    flush.fill_(1)
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        ev0.record(stream)
+        runner(steps)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1) / steps
+    gbs = 2.0 * n_el * esz / (ms / 1e3) / 1e9
+    out = {"config": desc, "ms_per_step": ms, "value": units / (ms / 1e3), "unit": unit,
+           "achieved_gbs": gbs, "frac_of_measured_peak": gbs / peak, "pct_of_8tbs": gbs / 8000.0,
+           "kernel": kern, "steps": steps, "clocks": clk.summary()}
+    del x
+    torch.cuda.empty_cache()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -457,6 +531,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-graph", action="store_true", help="launch each step from Python instead of a CUDA graph")
     ap.add_argument("--split", default=None, help="force the Schur split LO,HI (default: chosen at create)")
+    ap.add_argument("--extra", default=None,
+                    help="comma-separated workloads measured after the headline into extra_workloads "
+                         f"(default for the C2 run on one GPU: {EXTRA_DEFAULT}; 'none' to skip)")
     args = ap.parse_args()
     if args.workload in TWOD:
         if args.impl == "reference":
@@ -634,6 +711,16 @@ def main():
             "gpu_launches": args.steps,
             "cpu_baseline": cpu,
         }
+        extra = args.extra if args.extra is not None else (EXTRA_DEFAULT if (args.workload == "C2" and ws == 1) else "none")
+        if extra and extra != "none":
+            del x
+            torch.cuda.empty_cache()
+            line["extra_workloads"] = {}
+            for w in [e for e in extra.split(",") if e]:
+                try:
+                    line["extra_workloads"][w] = quick_measure(w)
+                except Exception as exc:  # report, do not lose the headline
+                    line["extra_workloads"][w] = {"error": f"{type(exc).__name__}: {exc}"}
         print(json.dumps(line), flush=True)
     if ws > 1:
         dist.destroy_process_group()
