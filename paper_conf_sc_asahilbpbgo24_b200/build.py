@@ -31,8 +31,9 @@ SOURCES = [
     ("warp_adv_f32.cu", "cu"),
     ("serial.cu", "cu"),
     ("refactor.cu", "cu"),
+    ("tile_pair_f64.cu", "cu"),
 ]
-HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh", "refactor.hpp"]
+HEADERS = ["host/plan.hpp", "device.hpp", "kernels.cuh", "refactor.hpp", "pair.cuh"]
 
 
 def _newer(target: str, deps: list[str]) -> bool:

@@ -78,6 +78,10 @@ struct KParams {
     int cbox;                        // rows of each corner box (0: corner reads the main tile)
     // dynamic shared memory offsets (bytes)
     int off_lw;                      // tile corner: Lambda window (DevPlan::lw_*)
+    // pair tile (pair.cuh): per CTA of the cluster: first row, rows, first segment,
+    // segments, boxes, and the arrivals that free each box
+    int pr_rb[2], pr_nrows[2], pr_seg0[2], pr_nseg[2], pr_nbox[2];
+    int pr_empty[2][NBOXMAX];
     int off_buf, off_L, off_U, off_dinv, off_G, off_H, off_fend, off_bbeg, off_x1, off_lamptr, off_lamc, off_lamv,
         off_gamr, off_gamc, off_gamv, off_gptr, off_dlu, off_dpiv, off_dscale, off_drow, off_mbar, off_cbuf,
         smem_total;

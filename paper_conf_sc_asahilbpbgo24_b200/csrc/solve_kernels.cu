@@ -7,6 +7,9 @@
 
 namespace sb {
 
+int launch_pair_f64(int K, const KParams &kp, const CUtensorMap *tm, int grid, int threads, cudaStream_t st, char *err,
+                    int errlen);
+
 // kernel chosen by the last launch_solve on this thread (spline_builder_last_kernel)
 static thread_local char g_last_kernel[96] = "";
 const char *last_kernel() { return g_last_kernel; }
@@ -42,7 +45,8 @@ int max_smem_of(int dev) {
     return v;
 }
 
-int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0) {
+int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t esz, size_t buf_bytes, int cbox = 0,
+                int fend_S = -1) {
     const size_t geo_bytes = (kp.adv && !P.adv_uniform) ? (size_t)GeoLayout(P).total_doubles * 8 : 0;
     size_t o = 0;
     auto take = [&](size_t bytes, size_t al) {
@@ -57,8 +61,9 @@ int layout_smem(KParams &kp, const DevPlan &P, const DevSeg &G, int R, size_t es
     kp.off_U = kp.off_dinv = kp.off_L;
     kp.off_G = take((size_t)S * K * K * esz, 16);
     kp.off_H = take((size_t)S * K * K * esz, 16);
-    kp.off_fend = take((size_t)S * R * K * esz, 16);
-    kp.off_bbeg = take((size_t)S * R * K * esz, 16);
+    const int FS = fend_S >= 0 ? fend_S : S;  // carry arrays: segments of this CTA (pair tile: half)
+    kp.off_fend = take((size_t)FS * R * K * esz, 16);
+    kp.off_bbeg = take((size_t)FS * R * K * esz, 16);
     kp.off_x1 = take((size_t)2 * R * k * esz, 16);
     kp.off_lamptr = take((size_t)(k + 1) * 4, 16);
     kp.off_lamc = take((size_t)P.lam_nnz * 4, 16);
@@ -220,6 +225,79 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((a.batch + 127) / 128, (int64_t)num_sms * 16));
         snprintf(g_last_kernel, sizeof(g_last_kernel), "serial<%s,K=%d>", a.dtype == 0 ? "f64" : "f32", P.K);
         return launch_serial(a.dtype, P.K, kp, grid, a.stream, err, errlen);
+    }
+    // pair tile (pair.cuh): 32-RHS tiles (256-B row chunks) split over a 2-CTA cluster.
+    // Worth it where the row pitch is large (C5: 8e6 RHS, 64 MB rows); SB_TILE_PAIR=0
+    // never, 2 whenever it applies (A/B), default 1: rows of at least pair_pitch bytes.
+    {
+        static const int pair_env = [] {
+            const char *e = getenv("SB_TILE_PAIR");
+            return e ? atoi(e) : 1;
+        }();
+        static const double pair_pitch = [] {
+            const char *e = getenv("SB_TILE_PAIR_PITCH_MB");
+            return (e ? atof(e) : 4.0) * 1048576.0;
+        }();
+        const DevSeg &G0 = P.seg[0];
+        const bool want = pair_env == 2 || (pair_env == 1 && (double)a.pstride * esz >= pair_pitch);
+        const int nseg0 = (G0.S + 1) / 2, nseg1 = G0.S - nseg0;
+        const int rb1 = P.s_lo + nseg0 * G0.L;  // first row of CTA 1
+        const bool fits_geom = G0.S >= 2 && nseg1 >= 1 && P.K <= 4 && P.k <= 8 && G0.LP == G0.L + 2 &&
+                               P.lw_head <= nseg0 * G0.L && P.nQ - P.lw_tail >= nseg0 * G0.L && rb1 < P.n;
+        const bool aligned = ((uintptr_t)a.rhs % 16 == 0) && ((a.pstride * (int64_t)esz) % 16 == 0) &&
+                             ((a.slab_stride * (int64_t)esz) % 16 == 0) && a.nslab < (1ll << 31);
+        if (want && a.dtype == 0 && fits_geom && aligned && a.batch >= 32 && get_encode()) {
+            KParams kp{};
+            kp.P = P;
+            kp.rhs = a.rhs;
+            kp.batch = a.batch;
+            kp.bstride = a.bstride;
+            kp.pstride = a.pstride;
+            kp.pr_rb[0] = 0; kp.pr_rb[1] = rb1;
+            kp.pr_nrows[0] = rb1; kp.pr_nrows[1] = P.n - rb1;
+            kp.pr_seg0[0] = 0; kp.pr_seg0[1] = nseg0;
+            kp.pr_nseg[0] = nseg0; kp.pr_nseg[1] = nseg1;
+            const int maxrows = std::max(kp.pr_nrows[0], kp.pr_nrows[1]);
+            const int nb = (maxrows + 255) / 256;
+            const int boxr = ((maxrows + nb - 1) / nb + 7) / 8 * 8;
+            kp.boxr = boxr;
+            for (int h = 0; h < 2; ++h) kp.pr_nbox[h] = (kp.pr_nrows[h] + boxr - 1) / boxr;
+            const int nbx = std::max(kp.pr_nbox[0], kp.pr_nbox[1]);
+            const int64_t tps = (a.batch + 31) / 32;
+            if (nbx <= NBOXMAX && tps * a.nslab < (1ll << 31) &&
+                layout_smem(kp, P, G0, 32, 8, (size_t)nbx * boxr * 32 * 8, (P.k + 1) / 2, nseg0) <= max_smem) {
+                kp.tps = (int)tps;
+                kp.ntiles = (int)(tps * a.nslab);
+                kp.slab_stride = a.slab_stride;
+                for (int h = 0; h < 2; ++h) {
+                    for (int c = 0; c < NBOXMAX; ++c) kp.pr_empty[h][c] = 1;  // unused boxes: any valid count
+                    for (int c = 0; c < kp.pr_nbox[h]; ++c) kp.pr_empty[h][c] = 1;  // the corner warp reads every box
+                    for (int sl = 0; sl < kp.pr_nseg[h]; ++sl) {
+                        const int sg = kp.pr_seg0[h] + sl, a0 = sg * G0.L;
+                        const int r0 = P.s_lo + a0 - kp.pr_rb[h];
+                        const int r1 = std::min(r0 + std::min(G0.L, P.nQ - a0), kp.pr_nrows[h]) - 1;
+                        for (int c = r0 / boxr; c <= r1 / boxr; ++c) kp.pr_empty[h][c]++;
+                    }
+                }
+                CUtensorMap tm[1];
+                memset(tm, 0, sizeof(tm));
+                cuuint64_t dims[3] = {(cuuint64_t)a.batch, (cuuint64_t)P.n, (cuuint64_t)a.nslab};
+                cuuint64_t strides[2] = {(cuuint64_t)(a.pstride * 8), (cuuint64_t)(a.slab_stride * 8)};
+                cuuint32_t box[3] = {32u, (cuuint32_t)boxr, 1u};
+                cuuint32_t estr[3] = {1, 1, 1};
+                CUresult cr = get_encode()(&tm[0], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, a.rhs, dims, strides, box, estr,
+                                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                if (cr != CUDA_SUCCESS) {
+                    snprintf(err, errlen, "cuTensorMapEncodeTiled (pair) failed (%d)", (int)cr);
+                    return 3;
+                }
+                const int threads = (std::max(nseg0, nseg1) + 1) * 32;
+                const int clusters = (int)std::min<int64_t>((int64_t)kp.ntiles, (int64_t)num_sms / 2);
+                snprintf(g_last_kernel, sizeof(g_last_kernel), "pair<f64,K=%d,R=32,TMA,2xCTA>", P.K);
+                return launch_pair_f64(P.K, kp, tm, 2 * clusters, threads, a.stream, err, errlen);
+            }
+        }
     }
     const DevSeg &G = P.seg[a.dtype == 0 ? 0 : 1];
     const int L = G.L;

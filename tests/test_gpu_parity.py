@@ -728,3 +728,43 @@ def test_update_device_faster_than_host_replan(torch_cuda):
     t_host = (time.perf_counter() - t0) / 5
     print(f"device update {t_dev * 1e3:.3f} ms, host re-plan {t_host * 1e3:.3f} ms")
     assert t_dev < t_host
+
+
+PAIR_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, %(root)r)
+import oracle
+from paper_conf_sc_asahilbpbgo24_b200 import SplineBuilder, inputs, last_kernel
+cases = [(3, 1000, 0, "uniform"), (5, 1000, 1, "sin"), (5, 996, 2, "sin"), (4, 1000, 0, "jitter"),
+         (3, 200, 1 | (2 << 4), "jitter"), (3, 1024, 0, "sin")]
+for deg, npts, bc, mesh in cases:
+    N = inputs.n_cells(deg, npts, bc)
+    x = inputs.breakpoints(N, mesh)
+    sb, o = SplineBuilder(deg, npts, bc, x), oracle.Oracle(deg, npts, bc, x)
+    for B in (32, 96, 32 * 74 * 2 + 6):
+        b = inputs.rhs(sb.n, B, seed=B, degree=deg, bc=bc)
+        t = torch.from_numpy(b).cuda()
+        sb.solve_(t)
+        torch.cuda.synchronize()
+        kern = last_kernel()
+        assert kern.startswith("pair<"), (deg, npts, bc, B, kern)
+        err = oracle.rel_coef_error(t.cpu().numpy(), o.solve(b))
+        assert err <= 1e-12, (deg, npts, bc, B, err)
+        assert o.residual(t.cpu().numpy(), b) <= 1e-12
+print("pair ok")
+"""
+
+
+def test_pair_tile_parity_forced(torch_cuda):
+    """The 2-CTA-cluster tile kernel (pair.cuh; 32-RHS tiles split in row halves,
+    carries and the corner exchanged through distributed shared memory) on
+    every band / boundary family, 1 to several tiles per cluster, forced with
+    SB_TILE_PAIR=2 in a subprocess (the dispatch reads it once per process)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SB_TILE_PAIR="2")
+    r = subprocess.run([sys.executable, "-c", PAIR_SCRIPT % {"root": root}], env=env, capture_output=True, text=True,
+                       timeout=300)
+    assert r.returncode == 0 and "pair ok" in r.stdout, r.stdout[-2000:] + r.stderr[-4000:]

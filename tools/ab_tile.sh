@@ -5,9 +5,9 @@
 O=gpurun_out/${O:-ab}
 mkdir -p $O
 for w in ${WL:-C2 C3G C3H}; do
-  python bench.py --workload $w --no-cpu-baseline --no-e2e > $O/main_$w.json 2> $O/main_$w.err
+  timeout ${BENCH_TIMEOUT:-180} python bench.py --workload $w --no-cpu-baseline --no-e2e > $O/main_$w.json 2> $O/main_$w.err
   for v in $LIBS; do
-    SB_LIB_PATH=$PWD/paper_conf_sc_asahilbpbgo24_b200/libsb_$v.so python bench.py --workload $w --no-cpu-baseline --no-e2e \
+    SB_LIB_PATH=$PWD/paper_conf_sc_asahilbpbgo24_b200/libsb_$v.so timeout ${BENCH_TIMEOUT:-180} python bench.py --workload $w --no-cpu-baseline --no-e2e \
       > $O/${v}_$w.json 2> $O/${v}_$w.err
   done
 done

@@ -128,30 +128,37 @@ static void run(double *x, int n, int64_t B, int sms, int boxr_req, CUtensorMapL
     printf("%-34s boxr=%3d mode=%d store=%d : %.3f ms  %.0f GB/s\n", tag, boxr, MODE, STORE, ms, bytes / ms / 1e6);
 }
 
-int main() {
-    const int n = 1000; const int64_t B = 100000;
+int main(int argc, char **argv) {
+    // argv[1]: batch B (row pitch = B doubles): 1e5 (C2, 800 KB) ... 8e6 (C5 on one GPU, 64 MB);
+    // argv[2] = "all": every variant, else the pitch study subset
+    const int n = 1000;
+    const int64_t B = argc > 1 ? (int64_t)atof(argv[1]) : 100000;
+    const bool all = argc > 2;
     int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
     double *x; CK(cudaMalloc(&x, (size_t)n * B * 8));
     CK(cudaMemset(x, 0, (size_t)n * B * 8));
+    printf("B = %lld (row pitch %.1f MB)\n", (long long)B, B * 8.0 / 1e6);
     auto P256 = CU_TENSOR_MAP_L2_PROMOTION_L2_256B, P128 = CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
          P0 = CU_TENSOR_MAP_L2_PROMOTION_NONE;
     run<3, 0>(x, n, B, sms, 256, P256, "rw st.cs prom256");
-    run<2, 3, 16, 2>(x, n, B, sms, 256, P256, "write only TMA store (R16 halves)");
-    run<3, 3, 16, 2>(x, n, B, sms, 256, P256, "rw TMA store (R16 halves)");
-    run<2, 3, 32, 4>(x, n, B, sms, 256, P256, "write only TMA store (R32 quarters)");
     run<3, 0, 32, 2>(x, n, B, sms, 256, P256, "R32 halves rw");
-    run<3, 0, 32, 2>(x, n, B, sms, 128, P256, "R32 halves rw box128");
-    run<1, 0, 32, 2>(x, n, B, sms, 256, P256, "R32 halves read only");
-    run<3, 0, 16, 2>(x, n, B, sms, 256, P256, "R16 halves rw (2 CTA/tile)");
-    run<3, 1>(x, n, B, sms, 256, P256, "rw st.wb prom256");
-    run<3, 2>(x, n, B, sms, 256, P256, "rw st.evict_first prom256");
-    run<3, 0>(x, n, B, sms, 256, P128, "rw st.cs prom128");
-    run<3, 0>(x, n, B, sms, 256, P0, "rw st.cs prom none");
-    run<3, 0>(x, n, B, sms, 128, P256, "rw st.cs box128");
-    run<3, 0>(x, n, B, sms, 64, P256, "rw st.cs box64");
     run<1, 0>(x, n, B, sms, 256, P256, "read only");
+    run<1, 0, 32, 2>(x, n, B, sms, 256, P256, "R32 halves read only");
     run<2, 0>(x, n, B, sms, 256, P256, "write only st.cs");
-    run<2, 1>(x, n, B, sms, 256, P256, "write only st.wb");
+    run<3, 3, 16, 2>(x, n, B, sms, 256, P256, "rw TMA store (R16 halves)");
+    if (all) {
+        run<2, 3, 16, 2>(x, n, B, sms, 256, P256, "write only TMA store (R16 halves)");
+        run<2, 3, 32, 4>(x, n, B, sms, 256, P256, "write only TMA store (R32 quarters)");
+        run<3, 0, 32, 2>(x, n, B, sms, 128, P256, "R32 halves rw box128");
+        run<3, 0, 16, 2>(x, n, B, sms, 256, P256, "R16 halves rw (2 CTA/tile)");
+        run<3, 1>(x, n, B, sms, 256, P256, "rw st.wb prom256");
+        run<3, 2>(x, n, B, sms, 256, P256, "rw st.evict_first prom256");
+        run<3, 0>(x, n, B, sms, 256, P128, "rw st.cs prom128");
+        run<3, 0>(x, n, B, sms, 256, P0, "rw st.cs prom none");
+        run<3, 0>(x, n, B, sms, 128, P256, "rw st.cs box128");
+        run<3, 0>(x, n, B, sms, 64, P256, "rw st.cs box64");
+        run<2, 1>(x, n, B, sms, 256, P256, "write only st.wb");
+    }
     CK(cudaFree(x));
     return 0;
 }
