@@ -54,6 +54,10 @@ struct spline_builder {
     cudaEvent_t rf_event = nullptr;
     bool rf_pending = false;
     double x0 = 0.0, xN = 1.0;    // periodic domain ends at create
+    // 2-D builder pipeline: pass 1 and pass 2 on two internal streams, chunk by chunk
+    std::mutex pipe_mu;
+    cudaStream_t pipe[2] = {nullptr, nullptr};
+    std::vector<cudaEvent_t> pipe_ev;
     // staging for solve_host
     std::mutex host_mu;
     void *stage[3] = {nullptr, nullptr, nullptr};
@@ -495,31 +499,73 @@ int spline_builder_solve_2d(spline_builder_t h1, spline_builder_t h2, void *rhs,
     if (batch > 1 && batch_stride < slice) return fail(SB_INVALID_ARG, "need batch_stride >= n1*n2");
     if (batch == 1) batch_stride = slice;
     const size_t esz = dtype == SB_F64 ? 8 : 4;
-    // Pass 1 (dim 1, contiguous rows) then pass 2 (dim 2, rows n1 apart).
-    // SB_2D_CHUNK_MB > 0 runs both passes chunk by chunk so a chunk is still in
-    // L2 when pass 2 reads it; measured on C6 (64 grids of 1024^2 fp64):
-    // unchunked 0.406 ms, 24 MB chunks 0.936, 96 MB 0.552 (launch tails), so the
-    // default is one chunk.
+    // Pass 1 (dim 1, contiguous rows) then pass 2 (dim 2, rows n1 apart), each one
+    // launch over every grid (default).  SB_2D_CHUNK_MB > 0: chunked pipeline -- pass 1
+    // of chunk c+1 on one internal stream while pass 2 of chunk c runs on the other
+    // (event per chunk; fork/join with the caller's stream, so graph capture works),
+    // so pass 2 would read a chunk pass 1 just left in L2.  Measured on C6 (64 grids
+    // of 1024^2 fp64): unchunked 0.369 ms; 16 / 32 / 48 / 96 MB chunks 0.751 / 0.577 /
+    // 0.502 / 0.448 ms -- every launch pays its pipeline fill and drain (constants
+    // staged, first tile loaded before any compute, last tile's compute not overlapped),
+    // which the L2 reuse does not repay (profiles/r02/ab_experiments.md).
     static const int64_t chunk_mb = [] {
         const char *e = getenv("SB_2D_CHUNK_MB");
-        return e ? (int64_t)atoll(e) : (int64_t)0;  // measured: chunked launches lose more to tails than L2 saves
+        return e ? (int64_t)atoll(e) : (int64_t)0;
     }();
+    auto pass1 = [&](void *base, int64_t nb, cudaStream_t st) {
+        if (batch_stride == slice) return do_solve(h1, base, dtype, nb * n2, n1, 1, st);
+        return do_solve(h1, base, dtype, n2, n1, 1, st, nullptr, nb, batch_stride);
+    };
+    auto pass2 = [&](void *base, int64_t nb, cudaStream_t st) {
+        return do_solve(h2, base, dtype, n1, 1, n1, st, nullptr, nb, batch_stride);
+    };
+    const cudaStream_t cs = (cudaStream_t)stream;
     int64_t cb = batch;
     if (chunk_mb > 0) cb = std::max<int64_t>(1, (chunk_mb << 20) / (slice * (int64_t)esz));
-    cb = std::min(cb, batch);
-    for (int64_t b0 = 0; b0 < batch; b0 += cb) {
-        const int64_t nb = std::min(cb, batch - b0);
-        void *base = (char *)rhs + (size_t)(b0 * batch_stride) * esz;
-        int st;
-        if (batch_stride == slice)
-            st = do_solve(h1, base, dtype, nb * n2, n1, 1, (cudaStream_t)stream);
-        else
-            st = do_solve(h1, base, dtype, n2, n1, 1, (cudaStream_t)stream, nullptr, nb, batch_stride);
-        if (st) return st;
-        st = do_solve(h2, base, dtype, n1, 1, n1, (cudaStream_t)stream, nullptr, nb, batch_stride);
-        if (st) return st;
+    if (cb >= batch) {  // one chunk: the two passes back to back on the caller's stream
+        int st = pass1(rhs, batch, cs);
+        if (!st) st = pass2(rhs, batch, cs);
+        return st;
     }
-    return SB_OK;
+    std::lock_guard<std::mutex> lock(h1->pipe_mu);
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != h1->device) cudaSetDevice(h1->device);
+    const int64_t nchunks = (batch + cb - 1) / cb;
+    auto bad = [&](cudaError_t e) {
+        if (cur != h1->device) cudaSetDevice(cur);
+        return fail(SB_CUDA, std::string("2-D pipeline: ") + cudaGetErrorString(e));
+    };
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < 2 && e == cudaSuccess; ++i)
+        if (!h1->pipe[i]) e = cudaStreamCreateWithFlags(&h1->pipe[i], cudaStreamNonBlocking);
+    while (e == cudaSuccess && (int64_t)h1->pipe_ev.size() < nchunks + 3) {
+        cudaEvent_t ev;
+        e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+        if (e == cudaSuccess) h1->pipe_ev.push_back(ev);
+    }
+    if (e != cudaSuccess) return bad(e);
+    cudaEvent_t *ev = h1->pipe_ev.data();  // [0] fork, [1] join A, [2] join B, [3 + c] pass 1 of chunk c done
+    const cudaStream_t sA = h1->pipe[0], sB = h1->pipe[1];
+    if ((e = cudaEventRecord(ev[0], cs)) != cudaSuccess) return bad(e);
+    if ((e = cudaStreamWaitEvent(sA, ev[0], 0)) != cudaSuccess || (e = cudaStreamWaitEvent(sB, ev[0], 0)) != cudaSuccess)
+        return bad(e);
+    int st = SB_OK;
+    for (int64_t c = 0; c < nchunks && !st; ++c) {
+        const int64_t b0 = c * cb, nb = std::min(cb, batch - b0);
+        void *base = (char *)rhs + (size_t)(b0 * batch_stride) * esz;
+        st = pass1(base, nb, sA);
+        if (st) break;
+        if ((e = cudaEventRecord(ev[3 + c], sA)) != cudaSuccess || (e = cudaStreamWaitEvent(sB, ev[3 + c], 0)) != cudaSuccess)
+            return bad(e);
+        st = pass2(base, nb, sB);
+    }
+    // join (also after a failed launch, so the caller's stream never runs ahead)
+    if ((e = cudaEventRecord(ev[1], sA)) != cudaSuccess || (e = cudaEventRecord(ev[2], sB)) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(cs, ev[1], 0)) != cudaSuccess || (e = cudaStreamWaitEvent(cs, ev[2], 0)) != cudaSuccess)
+        return bad(e);
+    if (cur != h1->device) cudaSetDevice(cur);
+    return st;
 }
 
 int spline_builder_solve_host(spline_builder_t h, void *host_rhs, int dtype, int64_t batch, int64_t ld) {
@@ -585,6 +631,9 @@ void spline_builder_destroy(spline_builder_t h) {
         if (h->device >= 0 && cur != h->device) cudaSetDevice(h->device);
         if (h->blob) cudaFree(h->blob);
         for (void *b : h->retired) cudaFree(b);
+        for (int i = 0; i < 2; ++i)
+            if (h->pipe[i]) cudaStreamDestroy(h->pipe[i]);
+        for (cudaEvent_t e : h->pipe_ev) cudaEventDestroy(e);
         if (h->stage_blob) cudaFree(h->stage_blob);
         if (h->rf_scratch) cudaFree(h->rf_scratch);
         if (h->rf_status) cudaFree(h->rf_status);
