@@ -75,6 +75,8 @@ struct KParams {
     int64_t slab_stride;             // tile kernel: elements between slabs of (n, batch) blocks
     int empty_count[NBOXMAX];        // arrivals that free box c (reader warps; corner warp if none)
     int corner_arrive_mask;          // boxes without a compute-warp reader: the corner warp frees them
+    int corner_need_mask;            // (no corner boxes) boxes holding the rows the corner reads
+    int box_order[NBOXMAX];          // TMA issue order of the boxes: the corner's boxes first
     int cbox;                        // rows of each corner box (0: corner reads the main tile)
     // dynamic shared memory offsets (bytes)
     int off_lw;                      // tile corner: Lambda window (DevPlan::lw_*)
@@ -626,7 +628,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             SB_TR(0);
             if (LOADER == LOAD_TMA) {
                 if (lane == 0) {
-                    for (int c = 0; c < nbox; ++c) {
+                    for (int q = 0; q < nbox; ++q) {
+                        const int c = p.box_order[q];  // the corner's boxes first: x1 starts earlier
                         if (it > 0) mbar_wait(empty + c, (it - 1) & 1);
                         mbar_arrive_expect_tx(full + c, box_bytes);
                         tma_load_3d(buf + (size_t)c * boxr * R, &tmap, full + c, tb * R, c * boxr, slab);
@@ -639,7 +642,8 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 SB_TR(8);
                 if (use_cbox) mbar_wait(cfull + (it & 1), (it >> 1) & 1);
                 else
-                    for (int c = 0; c < nbox; ++c) mbar_wait(full + c, it & 1);
+                    for (int c = 0; c < nbox; ++c)
+                        if ((p.corner_need_mask >> c) & 1) mbar_wait(full + c, it & 1);
             } else if (it > 0) {
                 mbar_wait(empty + 0, (it - 1) & 1);  // all compute warps finished tile it-1
             }
@@ -714,7 +718,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             if (lane == 0) {
                 if (LOADER == LOAD_TMA)
                     for (int c = 0; c < nbox; ++c)
-                        if (!use_cbox || ((p.corner_arrive_mask >> c) & 1)) mbar_arrive(empty + c);
+                        if ((p.corner_arrive_mask >> c) & 1) mbar_arrive(empty + c);
             }
         }
         return;
