@@ -464,7 +464,7 @@ template <typename C, typename T> struct CornerCtx {
     int part, lh, lw;
     const C *slw, *sdlu, *sdscale;
     const int *sdrow, *sdpiv;
-    C *sx1;            // this lane's x1 slot in shared memory
+    C *sx1;            // this lane's x1 slot in shared memory (x1[d] at sx1[d * R]: [d][rhs] order)
     T *gout;           // column of this RHS in HBM (nullptr: RHS beyond the batch)
     int64_t ps;
     const T *hb, *tb;  // b at the first row of the Lambda window's head / tail (this RHS)
@@ -516,7 +516,7 @@ __device__ __forceinline__ void tile_corner(const CornerCtx<C, T> &cx, LDB ldb) 
         for (int d = 0; d < KC; ++d) __stcs(cx.gout + (int64_t)cx.sdrow[d] * cx.ps, (T)xr[d]);
     if (cx.part == 0) {
 #pragma unroll
-        for (int d = 0; d < KC; ++d) cx.sx1[d] = xr[d];
+        for (int d = 0; d < KC; ++d) cx.sx1[d * R] = xr[d];
     }
 }
 
@@ -662,7 +662,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
             CornerCtx<C, T> cx;
             cx.part = part; cx.lh = P.lw_head; cx.lw = P.lw_head + P.lw_tail;
             cx.slw = slw; cx.sdlu = sdlu; cx.sdscale = sdscale; cx.sdrow = sdrow; cx.sdpiv = sdpiv;
-            cx.sx1 = sx1 + (it & 1) * R * k + rr * k;
+            cx.sx1 = sx1 + (it & 1) * R * k + rr;  // [d][rhs]: consecutive lanes, consecutive banks
             cx.gout = clive ? gs + ccol * p.bstride : nullptr; cx.ps = ps;
             {   // where the window rows of this RHS live: corner boxes, main tile or HBM
                 const int hr = s_lo, tr = s_lo + nQ - P.lw_tail;  // first rows of head / tail windows
@@ -787,7 +787,10 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         // ---------- b0 -= gamma x1 (only segments holding gamma rows wait for the corner warp)
         if (active && sgptr[s] < sgptr[s + 1]) {
             mbar_wait(x1full + (it & 1), (it >> 1) & 1);
-            const C *x1 = sx1 + (it & 1) * R * k + r0 * k;
+            // x1 order: [d][rhs] from the register corner (k <= 8, conflict-free), [rhs][d]
+            // from the shared-memory corner (k > 8)
+            const int xsr = k <= WCORNER_KREG ? 1 : k, xsd = k <= WCORNER_KREG ? R : 1;
+            const C *x1 = sx1 + (it & 1) * R * k + r0 * xsr;
             for (int e = sgptr[s]; e < sgptr[s + 1]; ++e) {
                 const int i = sgamr[e] - a;
                 const int dc = sgamc[e];
@@ -796,7 +799,7 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
                 for (int j = 0; j < L; ++j)
                     if (j == i)
 #pragma unroll
-                        for (int q = 0; q < NV; ++q) v[j][q] = fma(-gv, x1[q * k + dc], v[j][q]);
+                        for (int q = 0; q < NV; ++q) v[j][q] = fma(-gv, x1[q * xsr + dc * xsd], v[j][q]);
             }
         }
         SB_TR(2);

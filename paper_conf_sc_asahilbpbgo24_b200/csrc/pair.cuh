@@ -116,11 +116,11 @@ __device__ __forceinline__ void pair_corner(const KParams &p, int h, int it, int
     // exchange the partial vectors (double-buffered by tile parity)
     const int pb = (it & 1) * R * KC;
 #pragma unroll
-    for (int d = 0; d < KC; ++d) st_dsmem_f64(xpart_remote + (uint32_t)((pb + lane * KC + d) * 8), xr[d]);
+    for (int d = 0; d < KC; ++d) st_dsmem_f64(xpart_remote + (uint32_t)((pb + d * R + lane) * 8), xr[d]);
     mbar_arrive_remote(xready_remote + (uint32_t)((it & 1) * 8));  // the other CTA's xready[it & 1]
     PAIR_WAIT(xready + (it & 1), (it >> 1) & 1, "xready", it);
 #pragma unroll
-    for (int d = 0; d < KC; ++d) xr[d] += xpart[pb + lane * KC + d];
+    for (int d = 0; d < KC; ++d) xr[d] += xpart[pb + d * R + lane];
     wgetrs_reg<double, KC>(xr, sdlu, sdpiv, KC);
     if (gout)
 #pragma unroll
@@ -130,7 +130,7 @@ __device__ __forceinline__ void pair_corner(const KParams &p, int h, int it, int
             if (own) __stcs(gout + (int64_t)row * ps, xr[d]);
         }
 #pragma unroll
-    for (int d = 0; d < KC; ++d) sx1[lane * k + d] = xr[d];
+    for (int d = 0; d < KC; ++d) sx1[d * R + lane] = xr[d];  // [d][rhs]: conflict-free
 }
 
 template <int K, int L>
@@ -304,14 +304,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(TILE_MAX_THREADS, 1)
         // ---------- b0 -= gamma x1
         if (active && sgptr[s] < sgptr[s + 1]) {
             PAIR_WAIT(x1full + (it & 1), (it >> 1) & 1, "x1full", it);
-            const C *x1 = sx1 + (it & 1) * R * k + r0 * k;
+            const C *x1 = sx1 + (it & 1) * R * k + r0;  // [d][rhs]
             for (int e = sgptr[s]; e < sgptr[s + 1]; ++e) {
                 const int i = sgamr[e] - a;
                 const int dc = sgamc[e];
                 const C gv = sgamv[e];
 #pragma unroll
                 for (int j = 0; j < L; ++j)
-                    if (j == i) v[j][0] = fma(-gv, x1[dc], v[j][0]);
+                    if (j == i) v[j][0] = fma(-gv, x1[dc * R], v[j][0]);
             }
         }
         // ---------- local forward sweep, publish end state
