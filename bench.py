@@ -192,6 +192,13 @@ def dist_env():
     return ws, rank, local
 
 
+def use_dist(ws):
+    """NCCL process group (barrier + max-over-ranks timing) when there is more
+    than one rank; SB_BENCH_FORCE_DIST=1 takes the same path at world size 1
+    (exercises the NCCL code on a one-GPU box)."""
+    return ws > 1 or os.environ.get("SB_BENCH_FORCE_DIST") == "1"
+
+
 def make_rhs(deg, n, bc, B, first, layout, dtype):
     b = inputs.rhs(n, B, seed=1234, degree=deg, bc=bc, first=first)  # (n, B) fp64
     if layout == "point":
@@ -250,7 +257,7 @@ def run_2d(args):
     spec1, spec2, G, dt, desc = TWOD[args.workload]
     ws, rank, local = dist_env()
     torch.cuda.set_device(local)
-    if ws > 1:
+    if use_dist(ws):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     sbs = []
     for deg, npts, bc, mesh in (spec1, spec2):
@@ -265,7 +272,7 @@ def run_2d(args):
     stream = torch.cuda.current_stream()
 
     def barrier():
-        if ws > 1:
+        if use_dist(ws):
             dist.barrier()
         torch.cuda.synchronize()
 
@@ -298,7 +305,7 @@ def run_2d(args):
         barrier()
     total_ms = float(sum(s_.elapsed_time(e_) for s_, e_ in zip(starts, ends)))
     t_tensor = torch.tensor([total_ms], device="cuda", dtype=torch.float64)
-    if ws > 1:
+    if use_dist(ws):
         dist.all_reduce(t_tensor, op=dist.ReduceOp.MAX)
     ms_per_step = float(t_tensor[0]) / args.steps
     pts = n1 * n2 * G
@@ -320,7 +327,7 @@ def run_2d(args):
             torch.cuda.synchronize()
             ts.append(time.perf_counter() - t0)
         te = torch.tensor([float(np.mean(ts[1:]))], device="cuda", dtype=torch.float64)
-        if ws > 1:
+        if use_dist(ws):
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e = {"value": ws * pts / float(te[0]), "unit": "points/s", "h2d_bytes_per_step": int(host.nbytes),
                "d2h_bytes_per_step": int(host.nbytes), "path": "H2D + spline_builder_solve_2d + D2H"}
@@ -355,7 +362,7 @@ def run_2d(args):
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches_per_step * args.steps, "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
-    if ws > 1:
+    if use_dist(ws):
         dist.destroy_process_group()
 
 
@@ -549,7 +556,7 @@ def main():
 
     ws, rank, local = dist_env()
     torch.cuda.set_device(local)
-    if ws > 1:
+    if use_dist(ws):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     from paper_conf_sc_asahilbpbgo24_b200.shard import shard_bounds, weak_bounds
     deg, npts, bc, mesh, Bspec, dt, layout, desc = wl
@@ -585,7 +592,7 @@ def main():
         step = sb.solve_
 
     def barrier():
-        if ws > 1:
+        if use_dist(ws):
             dist.barrier()
         torch.cuda.synchronize()
 
@@ -622,7 +629,7 @@ def main():
     chunk_steps = [min(CHUNK, args.steps - c * CHUNK) for c in range(nchunks)]
     per_chunk = [s_.elapsed_time(e_) / m for s_, e_, m in zip(starts, ends, chunk_steps)]  # ms per step
     t_tensor = torch.tensor([total_ms, total_ms / args.steps], device="cuda", dtype=torch.float64)
-    if ws > 1:
+    if use_dist(ws):
         dist.all_reduce(t_tensor, op=dist.ReduceOp.MAX)
     total_ms, kern_avg_ms = float(t_tensor[0]), float(t_tensor[1])
     ms_per_step = total_ms / args.steps
@@ -649,7 +656,7 @@ def main():
                 sb.solve_host_(hp)
                 ts.append(time.perf_counter() - t0)
             te = torch.tensor([float(np.mean(ts))], device="cuda", dtype=torch.float64)
-            if ws > 1:
+            if use_dist(ws):
                 dist.all_reduce(te, op=dist.ReduceOp.MAX)
             e2e = {"value": ws * Be / float(te[0]), "unit": "RHS/s", "h2d_bytes_per_step": int(hsrc.nbytes),
                    "d2h_bytes_per_step": int(hsrc.nbytes), "path": "spline_builder_solve_host (pinned, chunked)",
@@ -667,7 +674,7 @@ def main():
                 torch.cuda.synchronize()
                 ts.append(time.perf_counter() - t0)
             te = torch.tensor([float(np.mean(ts[1:]))], device="cuda", dtype=torch.float64)
-            if ws > 1:
+            if use_dist(ws):
                 dist.all_reduce(te, op=dist.ReduceOp.MAX)
             e2e = {"value": ws * B / float(te[0]) * (n / 1e9 if adv else 1.0), "unit": "GLUPS" if adv else "RHS/s",
                    "h2d_bytes_per_step": int(hsrc.nbytes), "d2h_bytes_per_step": int(hsrc.nbytes),
@@ -722,7 +729,7 @@ def main():
                 except Exception as exc:  # report, do not lose the headline
                     line["extra_workloads"][w] = {"error": f"{type(exc).__name__}: {exc}"}
         print(json.dumps(line), flush=True)
-    if ws > 1:
+    if use_dist(ws):
         dist.destroy_process_group()
 
 

@@ -48,5 +48,14 @@ for mesh in ("sin", "jitter"):
     b = inputs.rhs(sb.n, 65, seed=7)
     sb.solve_(torch.from_numpy(b).cuda())
     sb.advect_(torch.from_numpy(b).cuda(), torch.linspace(-0.3, 0.7, 65, dtype=torch.float64).cuda())
+# device-side refactorisation (refactor + commit kernels), then solves on the new mesh
+for p, npts, bc in ((3, 1000, PERIODIC), (5, 1000, GREVILLE), (5, 996, HERMITE)):
+    N = inputs.n_cells(p, npts, bc)
+    sb = SplineBuilder(p, npts, bc, inputs.breakpoints(N, "sin"), device_update=True)
+    kn = torch.from_numpy(inputs.breakpoints(N, "jitter")).cuda()
+    sb.update_device_(kn)
+    sb.update_status()
+    b = inputs.rhs(sb.n, 40, seed=8, degree=p, bc=bc)
+    sb.solve_(torch.from_numpy(b).cuda())
 torch.cuda.synchronize()
 print("sanitize run done")
