@@ -581,8 +581,15 @@ int spline_builder_solve_host(spline_builder_t h, void *host_rhs, int dtype, int
     if (cur != h->device) cudaSetDevice(h->device);
     const size_t esz = dtype == SB_F64 ? 8 : 4;
     const int64_t n = h->plan.n;
-    // chunk of RHS per pipeline stage: ~64 MB, multiple of 16 columns
-    int64_t chunk = std::max<int64_t>(16, ((int64_t)(64ll << 20) / (n * (int64_t)esz)) / 16 * 16);
+    // chunk of RHS per pipeline stage: ~16 MB (SB_HOST_CHUNK_MB), multiple of 16 columns.
+    // Measured (C2, 800 + 800 MB per step over PCIe, whose copy ceiling is 16.1 ms):
+    // e2e 5.53-5.59e6 RHS/s at 16 MB vs 5.16e6 at 64 MB and 4.90e6 at 128 MB (shorter
+    // pipeline fill and drain); 4-12 MB were no better (profiles/r02/ab_experiments.md)
+    static const int64_t chunk_mb = [] {
+        const char *e = getenv("SB_HOST_CHUNK_MB");
+        return e && atoll(e) > 0 ? (int64_t)atoll(e) : (int64_t)16;
+    }();
+    int64_t chunk = std::max<int64_t>(16, ((int64_t)(chunk_mb << 20) / (n * (int64_t)esz)) / 16 * 16);
     chunk = std::min<int64_t>(chunk, (batch + 15) / 16 * 16);
     const size_t need = (size_t)chunk * n * esz;
     int rc = SB_OK;
