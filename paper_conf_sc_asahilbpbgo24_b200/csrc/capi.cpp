@@ -84,6 +84,15 @@ std::vector<C> conv(const std::vector<double> &v) {
     return std::vector<C>(v.begin(), v.end());
 }
 
+// [t][j][m] (host SegPlan) -> [j][m][t] (device; see upload)
+std::vector<double> seg_major(const std::vector<double> &M, int S, int K) {
+    std::vector<double> r(M.size(), 0.0);
+    for (int t = 0; t < S; ++t)
+        for (int j = 0; j < K; ++j)
+            for (int m = 0; m < K; ++m) r[((size_t)j * K + m) * S + t] = M[((size_t)t * K + j) * K + m];
+    return r;
+}
+
 int upload(spline_builder *h) {
     const sb::Plan &P = h->plan;
     const int K = P.K, nQ = P.nQ, k = P.k;
@@ -147,8 +156,15 @@ int upload(spline_builder *h) {
         }
         if (S > 0) gptr[S] = (int)P.gam_r.size();
         so[g].F[0] = pk.addv(F); so[g].F[1] = pk.addv(conv<float>(F));
-        so[g].G[0] = pk.addv(G.G); so[g].G[1] = pk.addv(conv<float>(G.G));
-        so[g].H[0] = pk.addv(G.H); so[g].H[1] = pk.addv(conv<float>(G.H));
+        // transfer matrices: the warp plan (g = 2) in [j][m][segment] order -- its lanes
+        // walk different segments, so consecutive lanes read consecutive words (the
+        // host plan's [segment][j][m] order made every K >= 2 walk load a 4- to 8-way
+        // bank conflict); the tile plans keep [segment][j][m] (two segments per warp,
+        // and the extra index arithmetic spilled the K = 3 tile kernel)
+        const std::vector<double> Gs = g == 2 ? seg_major(G.G, G.S, P.K) : G.G;
+        const std::vector<double> Hs = g == 2 ? seg_major(G.H, G.S, P.K) : G.H;
+        so[g].G[0] = pk.addv(Gs); so[g].G[1] = pk.addv(conv<float>(Gs));
+        so[g].H[0] = pk.addv(Hs); so[g].H[1] = pk.addv(conv<float>(Hs));
         so[g].gptr = pk.addv(gptr);
     }
     std::vector<double> rowf((size_t)std::max(nQ, 1) * (2 * K + 1), 0.0);

@@ -1237,7 +1237,7 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
                     C acc = __shfl_up_sync(0xffffffffu, st[j][0], w);
                     if (t >= 0)
 #pragma unroll
-                        for (int m = 0; m < K; ++m) acc = fma(sG[(t * K + j) * K + m], cin[m][0], acc);
+                        for (int m = 0; m < K; ++m) acc = fma(sG[(j * K + m) * S + t], cin[m][0], acc);
                     nw[j] = t >= 0 ? acc : C(0);
                 }
 #pragma unroll
@@ -1259,7 +1259,7 @@ __global__ void __launch_bounds__(32 * WARP_MAX_WARPS)
                     C acc = __shfl_down_sync(0xffffffffu, st[j][0], w);
                     if (t < S)
 #pragma unroll
-                        for (int m = 0; m < K; ++m) acc = fma(sH[(t * K + j) * K + m], co[m][0], acc);
+                        for (int m = 0; m < K; ++m) acc = fma(sH[(j * K + m) * S + t], co[m][0], acc);
                     nw[j] = t < S ? acc : C(0);
                 }
 #pragma unroll

@@ -390,6 +390,10 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
             const DevSeg &G = P.seg[g];
             if (G.S == 0) continue;
             const int L = G.L, Sg = G.S, LP = G.LP;
+            // transfer-matrix layout as in upload (capi.cpp): warp plan [j][m][t], tile plans [t][j][m]
+            auto gidx = [&](int t, int j, int m) -> size_t {
+                return g == 2 ? ((size_t)j * K + m) * Sg + t : ((size_t)t * K + j) * K + m;
+            };
             double *F8 = S8(G.F[0]);
             float *F4 = S4(G.F[1]);
             const size_t BS = (size_t)BW * LP;
@@ -428,11 +432,11 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
                         if (i >= L - K) last[L - 1 - i] = acc;
                     }
                     for (int j = 0; j < K; ++j) {
-                        G8[((size_t)t * K + j) * K + (m - 1)] = last[j];
-                        G4[((size_t)t * K + j) * K + (m - 1)] = (float)last[j];
+                        G8[gidx(t, j, m - 1)] = last[j];
+                        G4[gidx(t, j, m - 1)] = (float)last[j];
                     }
                 } else {
-                    for (int j = 0; j < K; ++j) { G8[(size_t)j * K + (m - 1)] = 0.0; G4[(size_t)j * K + (m - 1)] = 0.f; }
+                    for (int j = 0; j < K; ++j) { G8[gidx(0, j, m - 1)] = 0.0; G4[gidx(0, j, m - 1)] = 0.f; }
                 }
                 // backward: response of segment t to outflow unit m, at rows a+j
                 if (t + 1 < Sg) {
@@ -449,13 +453,13 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
                         if (i < K) first[i] = acc;
                     }
                     for (int j = 0; j < K; ++j) {
-                        H8[((size_t)t * K + j) * K + (m - 1)] = first[j];
-                        H4[((size_t)t * K + j) * K + (m - 1)] = (float)first[j];
+                        H8[gidx(t, j, m - 1)] = first[j];
+                        H4[gidx(t, j, m - 1)] = (float)first[j];
                     }
                 } else {
                     for (int j = 0; j < K; ++j) {
-                        H8[((size_t)t * K + j) * K + (m - 1)] = 0.0;
-                        H4[((size_t)t * K + j) * K + (m - 1)] = 0.f;
+                        H8[gidx(t, j, m - 1)] = 0.0;
+                        H4[gidx(t, j, m - 1)] = 0.f;
                     }
                 }
             }
@@ -470,7 +474,7 @@ __global__ void __launch_bounds__(256, 1) sb_refactor_kernel(const RefactorArgs 
                 double r = 0.0;
                 for (int j = 0; j < K; ++j) {
                     double sum = 0.0;
-                    for (int m = 0; m < K; ++m) sum += fabs(M[((size_t)t * K + j) * K + m]);
+                    for (int m = 0; m < K; ++m) sum += fabs(M[g == 2 ? ((size_t)j * K + m) * G.S + t : ((size_t)t * K + j) * K + m]);
                     r = fmax(r, sum);
                 }
                 return r;
