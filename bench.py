@@ -73,6 +73,9 @@ WORKLOADS = {
             "(1024, 2048) batch-contiguous blocks, spline_builder_solve_slabs), fp64"),
     "C5": (3, 1000, 0, "uniform", 8000000, "f64", "batch",
            "C5 cubic uniform periodic n=1000, 8e6 RHS in total sharded over the GPUs (strong scaling) fp64"),
+    "C5S8": (3, 1000, 0, "uniform", 1000000, "f64", "batch",
+             "C5's per-GPU shard at 8 GPUs (1e6 RHS, 8 MB row pitch) on one GPU: the per-GPU rate the "
+             "8-GPU strong-scaling run would see"),
 }
 
 
@@ -452,7 +455,7 @@ def run_reference(args, wl):
     print(json.dumps(line), flush=True)
 
 
-EXTRA_DEFAULT = "C1,C3G,C3H,C4,C4F32,C4M,ADV,ADVNU,C5,C6"
+EXTRA_DEFAULT = "C1,C3G,C3H,C4,C4F32,C4M,ADV,ADVNU,C5,C5S8,C6"
 
 
 def quick_measure(name, steps=20, warmup=3):
