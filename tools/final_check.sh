@@ -1,3 +1,6 @@
+#!/bin/bash
+# Round-end style check: pytest -m gpu, smoke, default bench, reference arm, torchrun line
+# through the NCCL path (SB_BENCH_FORCE_DIST=1), ncu launch list and one ncu --set full of C2
 O=gpurun_out/fin
 mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,clocks.mem,power.limit --format=csv > $O/gpu.txt 2>&1

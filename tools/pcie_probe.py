@@ -1,3 +1,4 @@
+"""PCIe copy ceiling: 800 MB pinned host <-> device, each direction alone and both at once."""
 import torch, time
 n = 800_000_000 // 8
 h1 = torch.empty(n, dtype=torch.float64).pin_memory(); h2 = torch.empty(n, dtype=torch.float64).pin_memory()
