@@ -133,6 +133,10 @@ int launch_warp(const DevPlan &P, const SolveArgs &a, int num_sms, int max_smem,
         const Cand &c = cands[ci];
         if (c.bulk && !can_bulk) continue;
         if (bulk_env >= 0 && c.bulk != (bulk_env > 0)) continue;
+        // the advection step with band K >= 2 runs better without the bulk pipeline
+        // (measured, Fig. 2 uniform p = 4 / 5: 0.592 -> 0.572 ms, 0.628 -> 0.609 ms;
+        // p = 3 (K = 1) keeps it: 0.373 vs 0.403 ms)
+        if (bulk_env < 0 && c.bulk && kp.adv && P.K >= 2) continue;
         KParams t = kp;
         layout_smem(t, P, G, 1, esz, (size_t)c.wpb * ((c.bulk ? 2 : 1) + out_row) * kp.wbuf_pitch * esz);
         if (t.smem_total > max_smem) continue;
