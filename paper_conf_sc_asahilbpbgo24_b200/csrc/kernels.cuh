@@ -851,12 +851,13 @@ __global__ void __launch_bounds__(TILE_MAX_THREADS, 1)
         named_bar(1, ncw * 32);  // B3: every local backward begin state is published
         SB_TR(6);
         // ---------- backward carry (true x at rows a+L..a+L+K-1) + correction chain
-        // TMA path, band K >= 2: every row is stored from inside the chain as soon as
-        // it is final (the last segment runs the chain with zero carries, so there is
-        // one store path).  Measured: C3 Greville 0.403 -> 0.380 ms, Hermite 0.335 ->
-        // 0.326 ms; for K = 1 (C2) the chain is too short to hide the stores and the
-        // burst after it is faster (0.285 vs 0.314 ms).
-        constexpr bool FUSED = LOADER == LOAD_TMA && NV == 1 && K >= 2;
+        // TMA path: every row is stored from inside the chain as soon as it is final
+        // (the last segment runs the chain with zero carries, so there is one store
+        // path).  Measured: C3 Greville 0.403 -> 0.380 ms, Hermite 0.335 -> 0.326 ms
+        // (round 1); band K = 1 took the burst after the chain until the round-2
+        // kernel, where the fused stores won too (C2 0.2888 -> 0.2866 ms, C4M 0.3752 ->
+        // 0.3724 ms, profiles/r02/ab_experiments.md).
+        constexpr bool FUSED = LOADER == LOAD_TMA && NV == 1;
         if (active && (FUSED || s < S - 1)) {
             C co[K][NV];
 #pragma unroll
