@@ -19,6 +19,26 @@ namespace {
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+// L2 promotion of the tile kernels' TMA loads.  Measured (same box, two rounds):
+// the single-CTA tile with band K = 1 (128-B row chunks) wants 256 B (C2 0.2832 vs
+// 0.2861 ms with 128 B or none); band K >= 2 and the pair tile (256-B chunks) want
+// none (C3 Greville 0.3159 vs 0.3178, C5S8 2.810 vs 2.853 ms).  SB_TILE_L2PROMO=0..3
+// (none, 64 B, 128 B, 256 B) overrides it for A/B runs.
+CUtensorMapL2promotion tile_l2_promotion(bool wide) {
+    static const int env = [] {
+        const char *e = getenv("SB_TILE_L2PROMO");
+        return e ? atoi(e) : -1;
+    }();
+    const int v = env >= 0 ? env : (wide ? 3 : 0);
+    switch (v) {
+        case 0: return CU_TENSOR_MAP_L2_PROMOTION_NONE;
+        case 1: return CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
+        case 2: return CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
+        default: return CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    }
+}
+
+
 // resolved once, thread-safe (C++11 magic static): concurrent first calls all
 // see the same result instead of racing on a half-written pointer
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -291,7 +311,7 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
                 cuuint32_t estr[3] = {1, 1, 1};
                 CUresult cr = get_encode()(&tm[0], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, a.rhs, dims, strides, box, estr,
                                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                                           tile_l2_promotion(false), CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
                 if (cr != CUDA_SUCCESS) {
                     snprintf(err, errlen, "cuTensorMapEncodeTiled (pair) failed (%d)", (int)cr);
                     return 3;
@@ -430,7 +450,7 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
             CUresult cr = get_encode()(&tm[q], a.dtype == 0 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64
                                                             : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
                                        3, a.rhs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                       CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                       CU_TENSOR_MAP_SWIZZLE_NONE, tile_l2_promotion(P.K == 1),
                                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             if (cr != CUDA_SUCCESS) {
                 snprintf(err, errlen, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
