@@ -338,7 +338,13 @@ int launch_solve(const DevPlan &P, const SolveArgs &a_in, int num_sms, char *err
     // TMA needs a 16-B aligned base, row pitch and slab pitch; boxes of <= 256 rows
     const bool aligned = ((uintptr_t)a.rhs % 16 == 0) && ((a.pstride * (int64_t)esz) % 16 == 0) &&
                          ((a.slab_stride * (int64_t)esz) % 16 == 0) && a.nslab < (1ll << 31);
-    const int nbox = (P.n + 255) / 256;
+    static const int box_max = [] {  // SB_TILE_BOXROWS: rows per TMA box at most (A/B; TMA limit 256)
+        const char *e = getenv("SB_TILE_BOXROWS");
+        const int v = e ? atoi(e) : 256;
+        return v >= 8 && v <= 256 ? v : 256;
+    }();
+    int nbox = (P.n + box_max - 1) / box_max;
+    if (nbox > NBOXMAX) nbox = (P.n + 255) / 256;
     const int boxr = ((P.n + nbox - 1) / nbox + 7) / 8 * 8;
     const int cands64[2] = {16, 8}, cands32[2] = {32, 16};
     const int *cands = a.dtype == 0 ? cands64 : cands32;
